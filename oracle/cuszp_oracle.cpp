@@ -1,0 +1,322 @@
+/*
+ * cuszp_oracle.cpp -- plain single-threaded C++17 oracle of the cuSZp
+ * compress / decompress path.  TEST INFRASTRUCTURE ONLY (see header).
+ *
+ * Written from the paper text, step by step, in the paper's order and
+ * notation (d_i data, r_i quantisation integers, l_i Lorenzo integers,
+ * F_k fixed length, CmpL_k block bytes).  No blocking, fusion or
+ * reordering beyond what the paper states.  Readings of ambiguous or
+ * garbled passages are DESIGN.md sec. 3, items R1..R12, cited as "R#".
+ *
+ * Build (kept deliberately plain; see __graft_entry__.build()):
+ *   g++ -std=c++17 -O2 -ffp-contract=off -fno-fast-math -shared -fPIC
+ * -ffp-contract=off keeps every float op a separately rounded IEEE op;
+ * the one fused multiply-add of the op sequence is an explicit fmaf().
+ */
+#include "cuszp_oracle.h"
+
+#include <cfenv>
+#include <cmath>
+#include <cstring>
+#include <vector>
+
+namespace {
+
+const int L = 32;                     /* block length, R1 */
+const int HEADER_BYTES = 32;          /* R10 */
+const float GUARD = 4194304.0f;       /* 2^22, R5 */
+const int MAX_F = 24;                 /* consequence of the guard, R5 */
+
+uint64_t align16(uint64_t v) { return (v + 15u) & ~uint64_t(15); }
+
+void put_u64(uint8_t* p, uint64_t v) { for (int i = 0; i < 8; ++i) p[i] = uint8_t(v >> (8 * i)); }
+uint64_t get_u64(const uint8_t* p) { uint64_t v = 0; for (int i = 0; i < 8; ++i) v |= uint64_t(p[i]) << (8 * i); return v; }
+void put_u32(uint8_t* p, uint32_t v) { for (int i = 0; i < 4; ++i) p[i] = uint8_t(v >> (8 * i)); }
+uint32_t get_u32(const uint8_t* p) { uint32_t v = 0; for (int i = 0; i < 4; ++i) v |= uint32_t(p[i]) << (8 * i); return v; }
+void put_f32(uint8_t* p, float f) { uint32_t u; std::memcpy(&u, &f, 4); put_u32(p, u); }
+float get_f32(const uint8_t* p) { uint32_t u = get_u32(p); float f; std::memcpy(&f, &u, 4); return f; }
+
+/* An absolute error bound is usable when eb and 2eb are positive, finite
+ * and normal (R5): 1/(2eb) is then finite. */
+bool eb_usable(float eb) {
+  if (!(eb >= 1.17549435e-38f)) return false;   /* FLT_MIN; rejects NaN, 0, <0 */
+  float two_eb = eb + eb;
+  return std::isfinite(two_eb);
+}
+
+/* Stream header, R10:
+ *  0 'CSZP' | 4 version=1 | 5 mode | 6 status | 7 log2(L)=5 | 8 u64 n |
+ * 16 f32 eb_abs | 20 f32 eb_in | 24 u64 payload_bytes                    */
+void write_header(uint8_t* out, uint64_t n, int mode, int status, float eb_abs,
+                  float eb_in, uint64_t payload_bytes) {
+  out[0] = 'C'; out[1] = 'S'; out[2] = 'Z'; out[3] = 'P';
+  out[4] = 1; out[5] = uint8_t(mode); out[6] = uint8_t(status); out[7] = 5;
+  put_u64(out + 8, n);
+  put_f32(out + 16, eb_abs);
+  put_f32(out + 20, eb_in);
+  put_u64(out + 24, payload_bytes);
+}
+
+/* Compression of x[0..n) with a resolved absolute bound eb_abs (sec 3.1,
+ * Fig 2): Quantisation and Prediction -> Fixed-length Encoding ->
+ * Global Synchronization -> Block Bit-shuffle. */
+int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int mode,
+                     uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  const uint64_t nb = (n + L - 1) / L;                  /* number of blocks N */
+  if (cap < oracle_max_compressed_bytes(n)) return ORACLE_ENOSPACE;
+  std::memset(out, 0, size_t(HEADER_BYTES + align16(nb)));
+
+  if (n == 0) {                                         /* R11 */
+    write_header(out, 0, mode, ORACLE_OK, eb_abs, eb_in, 0);
+    *out_bytes = HEADER_BYTES;
+    return ORACLE_OK;
+  }
+  if (!eb_usable(eb_abs)) {                             /* R5 */
+    write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0);
+    *out_bytes = HEADER_BYTES + align16(nb);
+    return ORACLE_ERANGE;
+  }
+
+  /* (1) Pre-quantisation, the only lossy step. */
+  std::vector<int32_t> r(static_cast<size_t>(nb * L), 0);            /* zero pad, R8 */
+  if (oracle_prequantize(x, size_t(n), eb_abs, r.data()) != ORACLE_OK) {
+    write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0);
+    *out_bytes = HEADER_BYTES + align16(nb);
+    return ORACLE_ERANGE;
+  }
+
+  /* (1') Lorenzo prediction inside each block. */
+  std::vector<int32_t> l(static_cast<size_t>(nb * L));
+  oracle_block_lorenzo(r.data(), size_t(nb), l.data());
+
+  /* (2) Fixed-length encoding: F_k and CmpL_k per block,
+   *     giving the BlockOffsetArray. */
+  std::vector<std::vector<uint8_t>> encoded(static_cast<size_t>(nb));
+  std::vector<uint64_t> block_offset(static_cast<size_t>(nb));
+  uint8_t* fixed_length = out + HEADER_BYTES;          /* Fig 12 part 1 */
+  for (uint64_t k = 0; k < nb; ++k) {
+    uint8_t buf[4 * (MAX_F + 1)];
+    int F = oracle_encode_block(&l[size_t(k * L)], buf);
+    fixed_length[k] = uint8_t(F);
+    block_offset[k] = oracle_block_bytes(F, L);
+    encoded[k].assign(buf, buf + block_offset[k]);
+  }
+
+  /* (3) Global synchronisation = exclusive prefix sum (Eq 3). */
+  std::vector<uint64_t> sync_offset(static_cast<size_t>(nb));
+  oracle_exclusive_scan(block_offset.data(), size_t(nb), sync_offset.data());
+  const uint64_t payload_bytes = sync_offset[nb - 1] + block_offset[nb - 1];
+
+  /* (4) Block bit-shuffled bytes placed at the synchronised offsets
+   *     (Fig 12 part 2). */
+  const uint64_t p0 = HEADER_BYTES + align16(nb);
+  for (uint64_t k = 0; k < nb; ++k)
+    if (block_offset[k] > 0)
+      std::memcpy(out + p0 + sync_offset[k], encoded[k].data(), size_t(block_offset[k]));
+
+  write_header(out, n, mode, ORACLE_OK, eb_abs, eb_in, payload_bytes);
+  *out_bytes = p0 + payload_bytes;
+  return ORACLE_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void oracle_value_range(const float* x, size_t n, float* mn, float* mx) {
+  /* r = max value - min value of the dataset.  A NaN anywhere
+   * makes the range undefined: both ends are reported as NaN (R5). */
+  float lo = INFINITY, hi = -INFINITY;
+  bool has_nan = false;
+  for (size_t i = 0; i < n; ++i) {
+    if (std::isnan(x[i])) { has_nan = true; continue; }
+    if (x[i] < lo) lo = x[i];
+    if (x[i] > hi) hi = x[i];
+  }
+  *mn = has_nan ? NAN : lo;
+  *mx = has_nan ? NAN : hi;
+}
+
+int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q) {
+  /* r_i = round(d_i / 2eb), guaranteeing |r_i * 2eb - d_i| <= eb.
+   * fp32 op sequence R2 (shared by definition, not by code, with the GPU):
+   *   two_eb = eb + eb; recip = 1 / two_eb           (once)
+   *   v  = d * recip                                   (RN)
+   *   r0 = rint(v)                                     (half-to-even)
+   *   res = fmaf(-r0, two_eb, d)   -- exact, see DESIGN R2
+   *   r  = r0 + (res > eb) - (res < -eb)   -> |d - r*2eb| <= eb exactly  */
+  std::fesetround(FE_TONEAREST);
+  const float two_eb = eb_abs + eb_abs;
+  const float recip = 1.0f / two_eb;
+  for (size_t i = 0; i < n; ++i) {
+    const float v = x[i] * recip;
+    if (!(std::fabs(v) < GUARD)) return ORACLE_ERANGE;  /* NaN/Inf/overflow, R5 */
+    const float r0 = std::nearbyint(v);
+    const float res = std::fmaf(-r0, two_eb, x[i]);
+    int32_t r = int32_t(r0);
+    if (res > eb_abs) r += 1;
+    else if (res < -eb_abs) r -= 1;
+    q[i] = r;
+  }
+  return ORACLE_OK;
+}
+
+void oracle_block_lorenzo(const int32_t* q, size_t nb, int32_t* l) {
+  /* l_i = r_i - r_{i-1}, r_{i-1} = 0 for the first integer of each block
+   * (P:525-529): the linear recurrence never crosses a block. */
+  for (size_t k = 0; k < nb; ++k) {
+    const int32_t* r = q + k * L;
+    int32_t* lk = l + k * L;
+    for (int i = 0; i < L; ++i) {
+      const int32_t prev = (i == 0) ? 0 : r[i - 1];
+      lk[i] = r[i] - prev;
+    }
+  }
+}
+
+int oracle_bit_length(uint32_t m) {
+  /* "the position of the last non-zero bit of this maximum integer"
+   * (P:566-568): 11 -> 4, 134 -> 8. */
+  int F = 0;
+  while (m != 0) { ++F; m >>= 1; }
+  return F;
+}
+
+uint64_t oracle_block_bytes(int F, int Lb) {
+  /* Eq 2: CmpL_k = (F_k + 1) * L / 8; a zero block stores nothing but
+   * its fixed-length byte (R6). */
+  if (F == 0) return 0;
+  return uint64_t(F + 1) * uint64_t(Lb) / 8;
+}
+
+void oracle_exclusive_scan(const uint64_t* cmpl, size_t k, uint64_t* sync_off) {
+  /* Eq 3: SyncOffsetArray = {0, CmpL_0, CmpL_0 + CmpL_1, ...}. */
+  uint64_t s = 0;
+  for (size_t i = 0; i < k; ++i) { sync_off[i] = s; s += cmpl[i]; }
+}
+
+int oracle_encode_block(const int32_t l[32], uint8_t* out) {
+  /* Sign map: bit 0 for positive, 1 otherwise; integer 0 -> bit 0 (R7).
+   * L/8 = 4 bytes; element j -> byte j/8, bit j%8 (R9). */
+  uint8_t sign_map[L / 8] = {0, 0, 0, 0};
+  uint32_t mag[L];
+  uint32_t max_abs = 0;
+  for (int j = 0; j < L; ++j) {
+    if (l[j] < 0) sign_map[j / 8] |= uint8_t(1u << (j % 8));
+    mag[j] = (l[j] < 0) ? uint32_t(-int64_t(l[j])) : uint32_t(l[j]);
+    if (mag[j] > max_abs) max_abs = mag[j];
+  }
+  /* Fixed length F = bit length of the block maximum. */
+  const int F = oracle_bit_length(max_abs);
+  if (F == 0) return 0;                                 /* zero block */
+  /* Block bit-shuffle: bit k of every |l_j| goes to the k-th
+   * group of L/8 bytes, after the sign map (R9). */
+  std::memcpy(out, sign_map, L / 8);
+  for (int k = 0; k < F; ++k) {
+    uint8_t* plane = out + (L / 8) * (1 + k);
+    for (int b = 0; b < L / 8; ++b) plane[b] = 0;
+    for (int j = 0; j < L; ++j)
+      if ((mag[j] >> k) & 1u) plane[j / 8] |= uint8_t(1u << (j % 8));
+  }
+  return F;
+}
+
+void oracle_decode_block(const uint8_t* payload, int F, int32_t l[32]) {
+  if (F == 0) { for (int j = 0; j < L; ++j) l[j] = 0; return; }
+  for (int j = 0; j < L; ++j) {
+    uint32_t mag = 0;
+    for (int k = 0; k < F; ++k) {
+      const uint8_t* plane = payload + (L / 8) * (1 + k);
+      if ((plane[j / 8] >> (j % 8)) & 1u) mag |= 1u << k;
+    }
+    const bool negative = (payload[j / 8] >> (j % 8)) & 1u;
+    l[j] = negative ? -int32_t(mag) : int32_t(mag);
+  }
+}
+
+uint64_t oracle_max_compressed_bytes(uint64_t n) {
+  const uint64_t nb = (n + L - 1) / L;
+  return HEADER_BYTES + align16(nb) + uint64_t(4 * (MAX_F + 1)) * nb;
+}
+
+int oracle_compress(const float* x, uint64_t n, float eb, int mode,
+                    uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr) return ORACLE_EINVAL;
+  if (mode == 0) {                                      /* ABS: eb = delta */
+    if (!eb_usable(eb)) return ORACLE_EINVAL;
+    return compress_with_eb(x, n, eb, eb, 0, out, cap, out_bytes);
+  }
+  if (mode == 1) {                                      /* REL: eb = lambda * r */
+    if (!(eb > 0.0f) || !std::isfinite(eb)) return ORACLE_EINVAL;
+    if (n == 0) return compress_with_eb(x, 0, 0.0f, eb, 1, out, cap, out_bytes);
+    float mn, mx;
+    oracle_value_range(x, size_t(n), &mn, &mx);
+    const float range = mx - mn;                        /* R3: fp32 */
+    const float eb_abs = eb * range;
+    return compress_with_eb(x, n, eb_abs, eb, 1, out, cap, out_bytes);
+  }
+  return ORACLE_EINVAL;
+}
+
+int oracle_compress_minmax(const float* x, uint64_t n, float lambda,
+                           const float* minmax, int n_pairs,
+                           uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr ||
+      minmax == nullptr || n_pairs <= 0) return ORACLE_EINVAL;
+  if (!(lambda > 0.0f) || !std::isfinite(lambda)) return ORACLE_EINVAL;
+  float mn = minmax[0], mx = minmax[1];
+  for (int p = 1; p < n_pairs; ++p) {
+    if (minmax[2 * p] < mn) mn = minmax[2 * p];
+    if (minmax[2 * p + 1] > mx) mx = minmax[2 * p + 1];
+  }
+  const float range = mx - mn;
+  const float eb_abs = lambda * range;
+  return compress_with_eb(x, n, eb_abs, lambda, 1, out, cap, out_bytes);
+}
+
+int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t n) {
+  /* Sec 3.2 / Fig 3: read the fixed lengths, rebuild CmpL (Eq 2), the same
+   * global synchronisation (Eq 3), then reverse bit-shuffle, fixed-length
+   * encoding and quantisation + prediction. */
+  if (in == nullptr || (n > 0 && out == nullptr)) return ORACLE_EINVAL;
+  if (in_bytes < uint64_t(HEADER_BYTES)) return ORACLE_ECORRUPT;
+  if (!(in[0] == 'C' && in[1] == 'S' && in[2] == 'Z' && in[3] == 'P') ||
+      in[4] != 1 || in[7] != 5) return ORACLE_ECORRUPT;
+  if (in[6] != ORACLE_OK) return in[6] == ORACLE_ERANGE ? ORACLE_ERANGE : ORACLE_ECORRUPT;
+  if (get_u64(in + 8) != n) return ORACLE_EINVAL;
+  if (n == 0) return ORACLE_OK;
+  const float eb_abs = get_f32(in + 16);
+  const uint64_t payload_bytes = get_u64(in + 24);
+  const uint64_t nb = (n + L - 1) / L;
+  const uint64_t p0 = HEADER_BYTES + align16(nb);
+  if (in_bytes < p0) return ORACLE_ECORRUPT;
+  if (!eb_usable(eb_abs)) return ORACLE_ECORRUPT;
+
+  const uint8_t* fixed_length = in + HEADER_BYTES;
+  std::vector<uint64_t> block_offset(static_cast<size_t>(nb));
+  for (uint64_t k = 0; k < nb; ++k) {
+    if (fixed_length[k] > MAX_F) return ORACLE_ECORRUPT;
+    block_offset[k] = oracle_block_bytes(fixed_length[k], L);
+  }
+  std::vector<uint64_t> sync_offset(static_cast<size_t>(nb));
+  oracle_exclusive_scan(block_offset.data(), size_t(nb), sync_offset.data());
+  const uint64_t total = sync_offset[nb - 1] + block_offset[nb - 1];
+  if (total != payload_bytes || in_bytes < p0 + total) return ORACLE_ECORRUPT;
+
+  const float two_eb = eb_abs + eb_abs;
+  for (uint64_t k = 0; k < nb; ++k) {
+    int32_t l[L];
+    oracle_decode_block(in + p0 + sync_offset[k], fixed_length[k], l);
+    /* reverse Lorenzo: r_i = r_{i-1} + l_i inside the block */
+    int32_t r = 0;
+    for (int i = 0; i < L; ++i) {
+      r += l[i];
+      const uint64_t idx = k * L + uint64_t(i);
+      /* d'_i = r_i * 2eb */
+      if (idx < n) out[idx] = float(r) * two_eb;
+    }
+  }
+  return ORACLE_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,99 @@
+/*
+ * cuszp_oracle.h -- plain, slow, single-threaded CPU oracle of cuSZp
+ * (Huang et al., SC'23, "cuSZp: An Ultra-fast GPU Error-bounded Lossy
+ * Compression Framework with Optimized End-to-End Performance").
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ * bench.py's cpu_baseline / --impl reference legs may load this library.
+ * The product path (paper_conf_sc_huangd0lc23_b200/) never links, imports
+ * or calls anything in oracle/, and this file shares no code, header,
+ * table or constant generator with the CUDA path.
+ *
+ * Citations: "P:NNN" = line NNN of the paper text with the
+ * section / equation / figure it falls in.  Readings of ambiguous passages
+ * are the ones listed in DESIGN.md section 3 ("Readings of the paper").
+ *
+ * Parity status: every function below is pinned by tests/test_oracle_*.py
+ * (golden blocks, closed forms, exact-arithmetic brute force, invariants);
+ * the only unpinned item is byte compatibility with the original, never
+ * released cuSZp binary ("parity unpinned" for that comparison).
+ */
+#ifndef CUSZP_ORACLE_H
+#define CUSZP_ORACLE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Status codes (same numeric meaning as the product ABI; written out
+ * independently here). */
+enum {
+  ORACLE_OK = 0,
+  ORACLE_EINVAL = 1,
+  ORACLE_ERANGE = 3,
+  ORACLE_ECORRUPT = 4,
+  ORACLE_ENOSPACE = 5
+};
+
+/* ---- individual steps of the method (each pinned on its own) ---------- */
+
+/* Eq 1 (sec 2.1): eb_abs = delta (ABS) or lambda * (max - min)
+ * (REL).  Writes exact min and max of x[0..n).  n must be > 0. */
+void oracle_value_range(const float* x, size_t n, float* mn, float* mx);
+
+/* Pre-quantisation r_i = round(d_i / 2eb) (sec 4.1).
+ * Writes q[0..n).  Returns ORACLE_OK or ORACLE_ERANGE (guard, DESIGN R5). */
+int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q);
+
+/* 1D 1-layer Lorenzo inside each L=32 block (sec 4.1):
+ * l_i = r_i - r_{i-1}, r_{-1} := 0 at every block start.  q and l have
+ * nb*32 entries (caller pads q with zeros past n, DESIGN R8). */
+void oracle_block_lorenzo(const int32_t* q, size_t nb, int32_t* l);
+
+/* "position of the last non-zero bit" of m (sec 4.2). */
+int oracle_bit_length(uint32_t m);
+
+/* Eq 2: CmpL = (F+1) * L / 8 bytes for a non-zero block,
+ * 0 for a zero block (DESIGN R6). */
+uint64_t oracle_block_bytes(int F, int L);
+
+/* Eq 3: exclusive prefix sum of the block offset array. */
+void oracle_exclusive_scan(const uint64_t* cmpl, size_t k, uint64_t* sync_off);
+
+/* Fixed-length encoding + block bit-shuffle of ONE block of 32 Lorenzo
+ * integers (sec 4.2, sec 4.4).  Returns F and writes
+ * CmpL = oracle_block_bytes(F, 32) payload bytes to out. */
+int oracle_encode_block(const int32_t l[32], uint8_t* out);
+
+/* Inverse of oracle_encode_block (sec 3.2). */
+void oracle_decode_block(const uint8_t* payload, int F, int32_t l[32]);
+
+/* ---- the whole path ---------------------------------------------------- */
+
+/* Largest stream for n elements: 32 + align16(nb) + 100 * nb. */
+uint64_t oracle_max_compressed_bytes(uint64_t n);
+
+/* Compress (sec 3.1, Fig 2).  mode 0 = ABS (eb is delta), 1 = REL (eb is
+ * lambda).  Writes the stream to out (capacity cap) and its length to
+ * *out_bytes.  Returns a status; on ORACLE_ERANGE the stream header carries
+ * status 3 and the payload is not meaningful. */
+int oracle_compress(const float* x, uint64_t n, float eb, int mode,
+                    uint8_t* out, uint64_t cap, uint64_t* out_bytes);
+
+/* REL compression of one shard against a global value range given as
+ * n_pairs (min, max) pairs (the sharded driver's contract). */
+int oracle_compress_minmax(const float* x, uint64_t n, float lambda,
+                           const float* minmax, int n_pairs,
+                           uint8_t* out, uint64_t cap, uint64_t* out_bytes);
+
+/* Decompress (sec 3.2, Fig 3).  n must equal the header's n. */
+int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out,
+                      uint64_t n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUSZP_ORACLE_H */
