@@ -1,0 +1,149 @@
+/*
+ * cuszp.h -- C ABI of the B200-native (sm_100a) cuSZp hot path.
+ *
+ * Method: Huang et al., "cuSZp: An Ultra-fast GPU Error-bounded Lossy
+ * Compression Framework with Optimized End-to-End Performance", SC'23.
+ * "P:NNN" cites line NNN of the paper text.  Readings of the
+ * paper (R1..R16) and the byte format are in DESIGN.md sections 3 and 4.
+ *
+ * Library: paper_conf_sc_huangd0lc23_b200/libcuszp.so (CUDA runtime linked
+ * statically).  Every symbol below is extern "C"; there are no C++ or torch
+ * types in any signature.  `stream` is a cudaStream_t passed as void*
+ * (NULL = legacy default stream).
+ *
+ * Conventions shared by all calls
+ * -------------------------------
+ *  - d_ pointers are CUDA device pointers, h_ pointers host pointers.
+ *  - The caller owns (allocates, frees) every buffer.  The asynchronous
+ *    calls never allocate, never synchronise and are CUDA-Graph capturable.
+ *  - Device buffers must be 16-byte aligned (d_in of compress: 4-byte).
+ *  - A workspace d_ws of cuszp_workspace_bytes(n) bytes must be ZEROED ONCE
+ *    when allocated (e.g. cudaMemset) and may then be reused for any number
+ *    of calls with element counts <= n.  Calls sharing a workspace must be
+ *    ordered (same stream, or event-ordered); concurrent calls need distinct
+ *    workspaces.
+ *  - Return value: CUSZP_OK, or a SYNCHRONOUS error detected on the host
+ *    (bad argument, too-small buffer, CUDA launch failure) -- nothing is
+ *    launched in that case.  DATA-DEPENDENT errors are ASYNCHRONOUS: they
+ *    are written to the stream header's status byte (compress) and to the
+ *    workspace; read them with cuszp_last_status() (synchronising).
+ */
+#ifndef CUSZP_H
+#define CUSZP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CUSZP_BLOCK_LEN 32      /* L, R1: pinned by Table 3's max CR 127.99 */
+#define CUSZP_HEADER_BYTES 32   /* R10 */
+#define CUSZP_VERSION 1
+
+typedef enum { CUSZP_ABS = 0, CUSZP_REL = 1 } cuszp_mode;
+
+typedef enum {
+  CUSZP_OK = 0,
+  CUSZP_EINVAL = 1,    /* bad argument (sync) / n != header n (async, decompress) */
+  CUSZP_ECUDA = 2,     /* CUDA error while launching or copying (sync) */
+  CUSZP_ERANGE = 3,    /* async: |d/2eb| >= 2^22, NaN/Inf data, unusable REL eb (R5) */
+  CUSZP_ECORRUPT = 4,  /* async: malformed stream (magic, F > 24, sizes, bounds) */
+  CUSZP_ENOSPACE = 5   /* sync: output or workspace too small */
+} cuszp_status;
+
+/* The 32-byte stream header, little-endian. */
+typedef struct {
+  char magic[4];           /* "CSZP" */
+  uint8_t version;         /* CUSZP_VERSION */
+  uint8_t mode;            /* cuszp_mode */
+  uint8_t status;          /* cuszp_status of the compression */
+  uint8_t log2_block_len;  /* 5 */
+  uint64_t n;              /* number of fp32 elements */
+  float eb_abs;            /* absolute bound used: delta (ABS) or lambda*(max-min) (REL, Eq 1) */
+  float eb_in;             /* user bound: delta (ABS) or lambda (REL) */
+  uint64_t payload_bytes;  /* sum of CmpL_k (Eq 2, Eq 3 total) */
+} cuszp_header;
+
+/* Largest stream for n elements: 32 + align16(ceil(n/32)) + 100*ceil(n/32)
+ * (F <= 24 by the R5 guard, so CmpL <= 4*25).  Output buffers of compress
+ * must be at least this large. */
+size_t cuszp_max_compressed_bytes(size_t n);
+
+/* Exact compressed size from the per-block fixed lengths F[0..nb) (host
+ * helper of Eq 2 + Eq 3): 32 + align16(nb) + sum_{F>0} 4(F+1). */
+size_t cuszp_compressed_bytes_from_F(const uint8_t* h_F, size_t nb);
+
+/* Workspace bytes for calls with up to n elements (look-back status words,
+ * tile ticket, range accumulators). */
+size_t cuszp_workspace_bytes(size_t n);
+
+/* a1 -- value range (Eq 1; R3, R4).  One kernel: 128-bit loads,
+ * warp/CTA reductions, one atomic per CTA on order-preserving integer keys;
+ * the last CTA writes (min, max) to d_minmax[0..1] (NaN if any NaN) and to
+ * the workspace.  d_minmax may be NULL.  n must be > 0. */
+int cuszp_range(const float* d_in, size_t n, float* d_minmax,
+                void* d_ws, size_t ws_bytes, void* stream);
+
+/* a1..a8 -- compression (sec 3.1, Fig 2; sec 4).  mode ABS: eb = delta;
+ * mode REL: eb = lambda and eb_abs = lambda*(max-min) is computed ON THE
+ * DEVICE (range kernel, then the fused compression kernel -- 2 launches;
+ * ABS: 1 launch).  Writes the stream to d_out and its
+ * exact length to *d_out_bytes (device u64, may be NULL).
+ * Sync errors: EINVAL (NULL pointers with n > 0, mode, eb <= 0 or
+ * non-finite, ABS eb not a normal float), ENOSPACE (out_capacity <
+ * cuszp_max_compressed_bytes(n), ws_bytes < cuszp_workspace_bytes(n)),
+ * ECUDA.  Async: ERANGE in the header status byte and the workspace. */
+int cuszp_compress(const float* d_in, size_t n, float eb, int mode,
+                   void* d_out, size_t out_capacity,
+                   unsigned long long* d_out_bytes,
+                   void* d_ws, size_t ws_bytes, void* stream);
+
+/* REL compression of one shard against a GLOBAL value range given on the
+ * device as n_pairs (min, max) float pairs (the sharded driver's NCCL
+ * all-gather result).  eb_abs = lambda*(max_p max -
+ * min_p min).  One launch. */
+int cuszp_compress_minmax(const float* d_in, size_t n, float lambda,
+                          const float* d_minmax, int n_pairs,
+                          void* d_out, size_t out_capacity,
+                          unsigned long long* d_out_bytes,
+                          void* d_ws, size_t ws_bytes, void* stream);
+
+/* a9..a12 -- decompression (sec 3.2, Fig 3): one fused kernel.  Reads the
+ * header on the device; n must equal the header's n (else async EINVAL).
+ * in_bytes bounds every read (corrupt offsets -> async ECORRUPT, nothing
+ * is read past d_in + in_bytes).  Writes d_out[0..n). */
+int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n,
+                     void* d_ws, size_t ws_bytes, void* stream);
+
+/* Status of the last compress/decompress call made with this workspace.
+ * SYNCHRONISES `stream`.  Returns a cuszp_status (or ECUDA). */
+int cuszp_last_status(const void* d_ws, void* stream);
+
+/* Copies the 32-byte header of a device stream to *h_hdr.  Synchronises. */
+int cuszp_read_header(const void* d_stream, cuszp_header* h_hdr, void* stream);
+
+/* End-to-end calls on HOST buffers (the e2e metric): H2D copy of the input,
+ * the device call, D2H of the result; synchronises before returning.
+ * Scratch device buffers are caller-owned (sizes as for the device calls);
+ * pinned host buffers give asynchronous copies.
+ * compress: h_out receives the stream, *h_out_bytes its exact length. */
+int cuszp_compress_host(const float* h_in, size_t n, float eb, int mode,
+                        void* h_out, size_t out_capacity, size_t* h_out_bytes,
+                        float* d_in_scratch, void* d_out_scratch,
+                        void* d_ws, size_t ws_bytes, void* stream);
+int cuszp_decompress_host(const void* h_in, size_t in_bytes, float* h_out, size_t n,
+                          void* d_in_scratch, float* d_out_scratch,
+                          void* d_ws, size_t ws_bytes, void* stream);
+
+/* Human-readable status name. */
+const char* cuszp_status_string(int status);
+
+/* CUSZP_VERSION * 100 + build id. */
+int cuszp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUSZP_H */

@@ -1,0 +1,207 @@
+"""paper_conf_sc_huangd0lc23_b200 -- B200-native cuSZp (Huang et al., SC'23).
+
+Thin Python binding over the C ABI in include/cuszp.h (libcuszp.so):
+argument marshalling only.  Every step of compression and decompression
+runs in the CUDA kernels of csrc/; torch supplies device memory, streams
+and (in .dist) process groups.  Tensors must be CUDA tensors: there is no
+CPU path.
+
+    import paper_conf_sc_huangd0lc23_b200 as cz
+    stream, nbytes = cz.compress(x, 1e-3, "rel")     # x: float32 CUDA tensor
+    y = cz.decompress(stream, x.numel())
+"""
+from __future__ import annotations
+
+import ctypes as C
+import struct
+
+import torch
+
+from ._lib import (  # noqa: F401
+    ECORRUPT, ECUDA, EINVAL, ENOSPACE, ERANGE, OK, STATUS_NAMES, CuszpError, check, lib,
+)
+
+ABS, REL = 0, 1
+HEADER_BYTES = 32
+BLOCK_LEN = 32
+
+__all__ = [
+    "ABS", "REL", "Workspace", "compress", "compress_minmax", "decompress", "value_range",
+    "max_compressed_bytes", "workspace_bytes", "last_status", "read_header", "compress_host",
+    "decompress_host", "CuszpError", "exact_bytes_from_F",
+]
+
+
+def _mode(mode) -> int:
+    if isinstance(mode, str):
+        return {"abs": ABS, "rel": REL}[mode.lower()]
+    return int(mode)
+
+
+def _stream_ptr(stream) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+def _require_cuda(t: torch.Tensor, name: str, dtype=None):
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor (no CPU path exists)")
+    if dtype is not None and t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+
+
+def max_compressed_bytes(n: int) -> int:
+    return int(lib().cuszp_max_compressed_bytes(int(n)))
+
+
+def workspace_bytes(n: int) -> int:
+    return int(lib().cuszp_workspace_bytes(int(n)))
+
+
+def exact_bytes_from_F(F) -> int:
+    import numpy as np
+
+    a = np.ascontiguousarray(F, dtype=np.uint8)
+    return int(lib().cuszp_compressed_bytes_from_F(a.ctypes.data_as(C.c_void_p), a.size))
+
+
+class Workspace:
+    """Zero-initialised device workspace for calls with up to ``n`` elements.
+    Calls sharing a workspace must be stream-ordered."""
+
+    def __init__(self, n: int, device=None):
+        device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        self.n = int(n)
+        self.nbytes = workspace_bytes(max(1, self.n))
+        self.buf = torch.zeros(self.nbytes, dtype=torch.uint8, device=device)
+
+    def ptr(self) -> int:
+        return self.buf.data_ptr()
+
+    def fits(self, n: int) -> bool:
+        return workspace_bytes(max(1, int(n))) <= self.nbytes
+
+
+_ws_cache: dict = {}
+
+
+def _workspace(n: int, device, ws: Workspace | None) -> Workspace:
+    if ws is not None:
+        if not ws.fits(n):
+            raise CuszpError(ENOSPACE, "workspace too small")
+        return ws
+    key = (device.index if device.index is not None else torch.cuda.current_device(), torch.cuda.current_stream(device).cuda_stream)
+    w = _ws_cache.get(key)
+    if w is None or not w.fits(n):
+        w = Workspace(max(int(n), 1 << 20), device)
+        _ws_cache[key] = w
+    return w
+
+
+def value_range(x: torch.Tensor, ws: Workspace | None = None, out: torch.Tensor | None = None, stream=None):
+    """(min, max) of x on the device as a float32 tensor of 2 (Eq 1's r)."""
+    _require_cuda(x, "x", torch.float32)
+    ws = _workspace(x.numel(), x.device, ws)
+    if out is None:
+        out = torch.empty(2, dtype=torch.float32, device=x.device)
+    check(lib().cuszp_range(x.data_ptr(), x.numel(), out.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
+          "cuszp_range")
+    return out
+
+
+def compress(x: torch.Tensor, eb: float, mode="rel", out: torch.Tensor | None = None,
+             out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None):
+    """Compress a float32 CUDA tensor.  Returns (stream buffer uint8 tensor of
+    capacity max_compressed_bytes(n), device int64 tensor [1] holding the
+    exact stream length).  Asynchronous; data errors land in the header."""
+    _require_cuda(x, "x", torch.float32)
+    n = x.numel()
+    cap = max_compressed_bytes(n)
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, device=x.device)
+    _require_cuda(out, "out", torch.uint8)
+    if out_bytes is None:
+        out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    ws = _workspace(n, x.device, ws)
+    check(lib().cuszp_compress(x.data_ptr(), n, float(eb), _mode(mode), out.data_ptr(), out.numel(),
+                               out_bytes.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_compress")
+    return out, out_bytes
+
+
+def compress_minmax(x: torch.Tensor, lam: float, minmax: torch.Tensor, out: torch.Tensor | None = None,
+                    out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None):
+    """REL compression against a global range given as (min, max) pairs on the device."""
+    _require_cuda(x, "x", torch.float32)
+    _require_cuda(minmax, "minmax", torch.float32)
+    n = x.numel()
+    if out is None:
+        out = torch.empty(max_compressed_bytes(n), dtype=torch.uint8, device=x.device)
+    if out_bytes is None:
+        out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    ws = _workspace(n, x.device, ws)
+    check(lib().cuszp_compress_minmax(x.data_ptr(), n, float(lam), minmax.data_ptr(), minmax.numel() // 2,
+                                      out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
+                                      _stream_ptr(stream)), "cuszp_compress_minmax")
+    return out, out_bytes
+
+
+def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None, in_bytes: int | None = None,
+               ws: Workspace | None = None, stream=None) -> torch.Tensor:
+    """Decompress a device stream into n float32 values (asynchronous)."""
+    _require_cuda(stream_buf, "stream_buf", torch.uint8)
+    if out is None:
+        out = torch.empty(int(n), dtype=torch.float32, device=stream_buf.device)
+    _require_cuda(out, "out", torch.float32)
+    ws = _workspace(n, stream_buf.device, ws)
+    nbytes = stream_buf.numel() if in_bytes is None else int(in_bytes)
+    check(lib().cuszp_decompress(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), ws.ptr(), ws.nbytes,
+                                 _stream_ptr(stream)), "cuszp_decompress")
+    return out
+
+
+def last_status(ws: Workspace | None = None, device=None, stream=None) -> int:
+    """Status of the last call on ``ws`` (synchronises the stream)."""
+    if ws is None:
+        device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        ws = _workspace(1, device, None)
+    return int(lib().cuszp_last_status(ws.ptr(), _stream_ptr(stream)))
+
+
+def read_header(stream_buf: torch.Tensor, stream=None) -> dict:
+    _require_cuda(stream_buf, "stream_buf", torch.uint8)
+    raw = (C.c_uint8 * 32)()
+    check(lib().cuszp_read_header(stream_buf.data_ptr(), C.cast(raw, C.c_void_p), _stream_ptr(stream)),
+          "cuszp_read_header")
+    b = bytes(raw)
+    n, = struct.unpack_from("<Q", b, 8)
+    eb_abs, eb_in = struct.unpack_from("<ff", b, 16)
+    payload, = struct.unpack_from("<Q", b, 24)
+    return dict(magic=b[:4], version=b[4], mode=b[5], status=b[6], log2l=b[7], n=n, eb_abs=eb_abs,
+                eb_in=eb_in, payload_bytes=payload)
+
+
+def compress_host(h_in, eb: float, mode, h_out, d_in_scratch: torch.Tensor, d_out_scratch: torch.Tensor,
+                  ws: Workspace, stream=None) -> int:
+    """End-to-end compression from a host float32 buffer (numpy or pinned
+    CPU tensor) into a host uint8 buffer; returns the stream length."""
+    n = h_in.numel() if isinstance(h_in, torch.Tensor) else h_in.size
+    pin = h_in.data_ptr() if isinstance(h_in, torch.Tensor) else h_in.ctypes.data
+    pout = h_out.data_ptr() if isinstance(h_out, torch.Tensor) else h_out.ctypes.data
+    cap = h_out.numel() if isinstance(h_out, torch.Tensor) else h_out.size
+    nbytes = C.c_size_t(0)
+    check(lib().cuszp_compress_host(pin, n, float(eb), _mode(mode), pout, cap, C.byref(nbytes),
+                                    d_in_scratch.data_ptr(), d_out_scratch.data_ptr(), ws.ptr(), ws.nbytes,
+                                    _stream_ptr(stream)), "cuszp_compress_host")
+    return int(nbytes.value)
+
+
+def decompress_host(h_in, in_bytes: int, h_out, d_in_scratch: torch.Tensor, d_out_scratch: torch.Tensor,
+                    ws: Workspace, stream=None) -> None:
+    n = h_out.numel() if isinstance(h_out, torch.Tensor) else h_out.size
+    pin = h_in.data_ptr() if isinstance(h_in, torch.Tensor) else h_in.ctypes.data
+    pout = h_out.data_ptr() if isinstance(h_out, torch.Tensor) else h_out.ctypes.data
+    check(lib().cuszp_decompress_host(pin, int(in_bytes), pout, n, d_in_scratch.data_ptr(),
+                                      d_out_scratch.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
+          "cuszp_decompress_host")

@@ -1,0 +1,263 @@
+// cuszp_abi.cu -- host side of the C ABI declared in include/cuszp.h:
+// argument validation, workspace / buffer sizing, persistent grid sizing,
+// kernel launches.  Never allocates, never synchronises (except the three
+// documented synchronous helpers), so every async call is graph-capturable.
+#include <cstring>
+#include <mutex>
+
+#include "internal.cuh"
+
+using namespace cuszp;
+
+namespace {
+
+uint64_t num_blocks(uint64_t n) { return (n + kL - 1) / kL; }
+uint64_t num_tiles(uint64_t n) { return (num_blocks(n) + kTileBlocks - 1) / kTileBlocks; }
+
+struct DeviceInfo {
+  int sms = 0;
+  int occ_compress = 0, occ_decompress = 0, occ_range = 0;
+};
+
+// Per-device launch geometry, computed once (occupancy of each kernel).
+int device_info(DeviceInfo* out) {
+  static std::mutex mu;
+  static DeviceInfo cache[64];
+  static bool have[64] = {false};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return CUSZP_ECUDA;
+  std::lock_guard<std::mutex> lock(mu);
+  if (!have[dev]) {
+    DeviceInfo d;
+    if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return CUSZP_ECUDA;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_compress, compress_kernel, kThreads, 0) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_decompress, decompress_kernel, kThreads, 0) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess)
+      return CUSZP_ECUDA;
+    cache[dev] = d;
+    have[dev] = true;
+  }
+  *out = cache[dev];
+  return CUSZP_OK;
+}
+
+bool eb_is_normal(float eb) {
+  if (!(eb >= kFltMin)) return false;
+  const float two = eb + eb;
+  return two - two == 0.0f;   // finite
+}
+
+uint32_t status_capacity(size_t ws_bytes) {
+  const uint64_t c = (ws_bytes - kWsCtrlBytes) / 8;
+  return c > 0xffffffffull ? 0xffffffffu : uint32_t(c);
+}
+
+int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const float* d_minmax,
+                    int n_pairs, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
+                    void* d_ws, size_t ws_bytes, cudaStream_t stream) {
+  if (out_capacity < cuszp_max_compressed_bytes(n) || ws_bytes < cuszp_workspace_bytes(n))
+    return CUSZP_ENOSPACE;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  CompressArgs a;
+  a.in = d_in;
+  a.n = n;
+  a.nb = num_blocks(n);
+  a.num_tiles = uint32_t(num_tiles(n));
+  a.mode = mode;
+  a.eb_in = eb_in;
+  a.minmax = d_minmax;
+  a.n_pairs = n_pairs;
+  a.out = static_cast<uint8_t*>(d_out);
+  a.out_bytes = d_out_bytes;
+  a.ws = static_cast<WsCtrl*>(d_ws);
+  a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
+  a.status_cap = status_capacity(ws_bytes);
+  uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_compress > 0 ? di.occ_compress : 1);
+  if (grid > a.num_tiles) grid = a.num_tiles;
+  if (grid < 1) grid = 1;
+  compress_kernel<<<unsigned(grid), kThreads, 0, stream>>>(a);
+  return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+}
+
+}  // namespace
+
+extern "C" {
+
+size_t cuszp_max_compressed_bytes(size_t n) {
+  const uint64_t nb = num_blocks(n);
+  return size_t(kHdr + align16(nb) + uint64_t(4 * (kMaxF + 1)) * nb);
+}
+
+size_t cuszp_compressed_bytes_from_F(const uint8_t* h_F, size_t nb) {
+  uint64_t s = kHdr + align16(nb);
+  for (size_t k = 0; k < nb; ++k)
+    if (h_F[k]) s += 4u * (uint64_t(h_F[k]) + 1u);
+  return size_t(s);
+}
+
+size_t cuszp_workspace_bytes(size_t n) {
+  const uint64_t t = num_tiles(n);
+  return size_t(kWsCtrlBytes + 8 * (t > 0 ? t : 1));
+}
+
+int cuszp_range(const float* d_in, size_t n, float* d_minmax, void* d_ws, size_t ws_bytes, void* stream) {
+  if (d_in == nullptr || d_ws == nullptr || n == 0 || (reinterpret_cast<uintptr_t>(d_in) & 3u))
+    return CUSZP_EINVAL;
+  if (ws_bytes < kWsCtrlBytes) return CUSZP_ENOSPACE;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  RangeArgs a{d_in, n, d_minmax, static_cast<WsCtrl*>(d_ws)};
+  const uint64_t want = (n / 4 + 255) / 256;   // one float4 per thread at most
+  uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_range > 0 ? di.occ_range : 1);
+  if (grid > want) grid = want;
+  if (grid < 1) grid = 1;
+  range_kernel<<<unsigned(grid), 256, 0, static_cast<cudaStream_t>(stream)>>>(a);
+  return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+}
+
+int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out, size_t out_capacity,
+                   unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes, void* stream) {
+  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr) return CUSZP_EINVAL;
+  if ((reinterpret_cast<uintptr_t>(d_in) & 3u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
+      (reinterpret_cast<uintptr_t>(d_ws) & 15u))
+    return CUSZP_EINVAL;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (mode == CUSZP_ABS) {
+    if (!eb_is_normal(eb)) return CUSZP_EINVAL;
+    return launch_compress(d_in, n, CUSZP_ABS, eb, nullptr, 0, d_out, out_capacity, d_out_bytes, d_ws,
+                           ws_bytes, s);
+  }
+  if (mode == CUSZP_REL) {
+    if (!(eb > 0.0f) || !(eb - eb == 0.0f)) return CUSZP_EINVAL;
+    if (out_capacity < cuszp_max_compressed_bytes(n) || ws_bytes < cuszp_workspace_bytes(n))
+      return CUSZP_ENOSPACE;
+    const WsCtrl* ws = static_cast<const WsCtrl*>(d_ws);
+    if (n > 0) {
+      const int st = cuszp_range(d_in, n, nullptr, d_ws, ws_bytes, stream);
+      if (st != CUSZP_OK) return st;
+    }
+    return launch_compress(d_in, n, CUSZP_REL, eb, ws->minmax, 1, d_out, out_capacity, d_out_bytes,
+                           d_ws, ws_bytes, s);
+  }
+  return CUSZP_EINVAL;
+}
+
+int cuszp_compress_minmax(const float* d_in, size_t n, float lambda, const float* d_minmax, int n_pairs,
+                          void* d_out, size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws,
+                          size_t ws_bytes, void* stream) {
+  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || d_minmax == nullptr ||
+      n_pairs <= 0)
+    return CUSZP_EINVAL;
+  if ((reinterpret_cast<uintptr_t>(d_in) & 3u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
+      (reinterpret_cast<uintptr_t>(d_ws) & 15u))
+    return CUSZP_EINVAL;
+  if (!(lambda > 0.0f) || !(lambda - lambda == 0.0f)) return CUSZP_EINVAL;
+  return launch_compress(d_in, n, CUSZP_REL, lambda, d_minmax, n_pairs, d_out, out_capacity, d_out_bytes,
+                         d_ws, ws_bytes, static_cast<cudaStream_t>(stream));
+}
+
+int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n, void* d_ws, size_t ws_bytes,
+                     void* stream) {
+  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr) return CUSZP_EINVAL;
+  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 3u) ||
+      (reinterpret_cast<uintptr_t>(d_ws) & 15u))
+    return CUSZP_EINVAL;
+  if (ws_bytes < cuszp_workspace_bytes(n)) return CUSZP_ENOSPACE;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  DecompressArgs a;
+  a.in = static_cast<const uint8_t*>(d_in);
+  a.in_bytes = in_bytes;
+  a.out = d_out;
+  a.n = n;
+  a.nb = num_blocks(n);
+  a.num_tiles = uint32_t(num_tiles(n));
+  a.ws = static_cast<WsCtrl*>(d_ws);
+  a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
+  a.status_cap = status_capacity(ws_bytes);
+  uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_decompress > 0 ? di.occ_decompress : 1);
+  if (grid > a.num_tiles) grid = a.num_tiles;
+  if (grid < 1) grid = 1;
+  decompress_kernel<<<unsigned(grid), kThreads, 0, static_cast<cudaStream_t>(stream)>>>(a);
+  return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+}
+
+int cuszp_last_status(const void* d_ws, void* stream) {
+  if (d_ws == nullptr) return CUSZP_EINVAL;
+  uint32_t st = 0;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (cudaMemcpyAsync(&st, &static_cast<const WsCtrl*>(d_ws)->last_status, 4, cudaMemcpyDeviceToHost, s) !=
+          cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  return int(st);
+}
+
+int cuszp_read_header(const void* d_stream, cuszp_header* h_hdr, void* stream) {
+  if (d_stream == nullptr || h_hdr == nullptr) return CUSZP_EINVAL;
+  static_assert(sizeof(cuszp_header) == 32, "header layout");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (cudaMemcpyAsync(h_hdr, d_stream, 32, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  return CUSZP_OK;
+}
+
+int cuszp_compress_host(const float* h_in, size_t n, float eb, int mode, void* h_out, size_t out_capacity,
+                        size_t* h_out_bytes, float* d_in_scratch, void* d_out_scratch, void* d_ws,
+                        size_t ws_bytes, void* stream) {
+  if ((n > 0 && (h_in == nullptr || d_in_scratch == nullptr)) || h_out == nullptr || h_out_bytes == nullptr ||
+      d_out_scratch == nullptr)
+    return CUSZP_EINVAL;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (n > 0 && cudaMemcpyAsync(d_in_scratch, h_in, n * sizeof(float), cudaMemcpyHostToDevice, s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  // the exact length lands in the workspace's pad area (device u64)
+  unsigned long long* d_len =
+      reinterpret_cast<unsigned long long*>(&static_cast<WsCtrl*>(d_ws)->pad[2]);
+  int st = cuszp_compress(d_in_scratch, n, eb, mode, d_out_scratch, cuszp_max_compressed_bytes(n), d_len, d_ws,
+                          ws_bytes, stream);
+  if (st != CUSZP_OK) return st;
+  unsigned long long len = 0;
+  if (cudaMemcpyAsync(&len, d_len, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  if (len > out_capacity) return CUSZP_ENOSPACE;
+  if (cudaMemcpyAsync(h_out, d_out_scratch, size_t(len), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  *h_out_bytes = size_t(len);
+  return CUSZP_OK;
+}
+
+int cuszp_decompress_host(const void* h_in, size_t in_bytes, float* h_out, size_t n, void* d_in_scratch,
+                          float* d_out_scratch, void* d_ws, size_t ws_bytes, void* stream) {
+  if (h_in == nullptr || d_in_scratch == nullptr || (n > 0 && (h_out == nullptr || d_out_scratch == nullptr)))
+    return CUSZP_EINVAL;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (cudaMemcpyAsync(d_in_scratch, h_in, in_bytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  int st = cuszp_decompress(d_in_scratch, in_bytes, d_out_scratch, n, d_ws, ws_bytes, stream);
+  if (st != CUSZP_OK) return st;
+  if (n > 0 && cudaMemcpyAsync(h_out, d_out_scratch, n * sizeof(float), cudaMemcpyDeviceToHost, s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  if (cudaStreamSynchronize(s) != cudaSuccess) return CUSZP_ECUDA;
+  return CUSZP_OK;
+}
+
+const char* cuszp_status_string(int status) {
+  switch (status) {
+    case CUSZP_OK: return "CUSZP_OK";
+    case CUSZP_EINVAL: return "CUSZP_EINVAL";
+    case CUSZP_ECUDA: return "CUSZP_ECUDA";
+    case CUSZP_ERANGE: return "CUSZP_ERANGE";
+    case CUSZP_ECORRUPT: return "CUSZP_ECORRUPT";
+    case CUSZP_ENOSPACE: return "CUSZP_ENOSPACE";
+    default: return "CUSZP_UNKNOWN";
+  }
+}
+
+int cuszp_version(void) { return CUSZP_VERSION * 100 + 1; }
+
+}  // extern "C"
