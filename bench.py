@@ -1,0 +1,387 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of the cuSZp hot path on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl ours|reference]
+                    [--config c2_hurricane|c1_smooth1d|c3_hacc|c4_nyx|c5_rtm]
+
+A STEP is one pass of the whole hot path over one
+batch of synthetic input: for every field of the config and every REL error
+bound it names, value range (a1) -> fused compression (a2..a8) -> fused
+decompression (a9..a12), all through the C ABI.  The default workload is
+BASELINE configs[1]: three Hurricane-shaped 100x500x500 fp32 fields (U,
+QCLOUD, TC) at REL 1e-2, 1e-3, 1e-4 -> 9 round trips, 900 MB of fp32 input
+per step per GPU.
+
+Timing: the L2 (126 MB) is flushed (a 512 MB write, untimed) before every
+round trip; each round trip is bracketed by CUDA events on the launching
+stream; a step's time is the sum of its round trips' device time.  W warm-up
+steps, then K timed steps between barrier + synchronize; max over ranks.
+Multi-GPU (torchrun): weak scaling -- every rank compresses its own fields
+with the GLOBAL REL range (NCCL all-gather of (min,max)) and all-gathers the
+compressed byte counts to build the container header (paper_conf_sc_
+huangd0lc23_b200.dist).
+
+--impl reference runs the CPU oracle (oracle/, single thread) on a bounded
+sample of the same config -- the tier's reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+PAPER_A100 = {"compress_mean_gbs": 93.63, "decompress_mean_gbs": 120.04,
+              "source": "PAPER.md P:961-962 (A100 40GB, real SDRBench data, REL 1E-1..1E-4)"}
+FALLBACK_HBM_GBS = 6650.0
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--config", default="c2_hurricane")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=10.0)
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------ helpers
+
+def peak_hbm():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 100 ms while running."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines: list[str] = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                smax = float(parts[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        loaded = [s for s in sm if smax and s > 0.5 * smax] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def workload(cfg_name: str):
+    import synth
+
+    c = synth.CONFIGS[cfg_name]
+    fields = c.get("fields", [None])
+    return c, fields, c["rel"]
+
+
+# ---------------------------------------------------------------- reference arm
+
+def run_reference(args, rank, world):
+    """The CPU oracle, as it stands, on a bounded sample of the same config."""
+    if rank != 0:
+        return
+    import oracle
+    import synth
+
+    oracle.build()
+    c, fields, rels = workload(args.config)
+    x = synth.field_for_config(args.config, device="cpu", field=fields[0]).numpy()
+    sample = x[: min(x.size, 1 << 22)].copy()
+    rel = rels[len(rels) // 2]
+    t_steps = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        st, s = oracle.compress(sample, rel, oracle.REL)
+        st2, y = oracle.decompress(s, sample.size)
+        dt = time.perf_counter() - t0
+        assert st == st2 == oracle.OK
+        if i >= args.warmup:
+            t_steps.append(dt)
+    tot = sum(t_steps)
+    gbs = sample.size * 4 * len(t_steps) / tot / 1e9
+    line = {
+        "impl": "reference", "metric": "end-to-end compress+decompress GB/s (input fp32)", "value": gbs,
+        "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": tot / len(t_steps) * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": args.config, "field": fields[0], "rel": rel, "n": int(sample.size),
+                   "sample": f"first {sample.size} elements of the {args.config} field"},
+        "cpu_baseline": {"value": gbs, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{sample.size} elements ({sample.size * 4 / 1e6:.1f} MB) of {args.config}/{fields[0]} at REL {rel}, one round trip per step"},
+        "e2e": {"value": gbs, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# -------------------------------------------------------------------- our arm
+
+def cpu_baseline(args, cfg_name, fields, rels):
+    import oracle
+    import synth
+
+    oracle.build()
+    x = synth.field_for_config(cfg_name, device="cpu", field=fields[0]).numpy()
+    rel = rels[len(rels) // 2]
+    n_done, t_tot, reps = 0, 0.0, 0
+    while t_tot < args.cpu_seconds or reps == 0:
+        t0 = time.perf_counter()
+        st, s = oracle.compress(x, rel, oracle.REL)
+        st2, y = oracle.decompress(s, x.size)
+        t_tot += time.perf_counter() - t0
+        n_done += x.size
+        reps += 1
+    return {"value": n_done * 4 / t_tot / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"{reps} round trip(s) of {cfg_name}/{fields[0]} ({x.size} elements) at REL {rel}, "
+                      f"{t_tot:.1f} s single-threaded C++ oracle"}
+
+
+def run_ours(args, rank, world, dev):
+    import paper_conf_sc_huangd0lc23_b200 as cz
+    import synth
+    from paper_conf_sc_huangd0lc23_b200 import dist as czd
+
+    lib = cz.lib()
+    c, fields, rels = workload(args.config)
+    stream = torch.cuda.current_stream(dev)
+    sp = int(stream.cuda_stream)
+
+    # ---- inputs resident in HBM (generated on the device, seeded per rank)
+    xs = {}
+    for f in fields:
+        xs[f] = synth.field_for_config(args.config, device=dev, field=f)
+        if world > 1 and rank > 0:
+            xs[f] = xs[f].roll(rank * 4099)      # distinct data per rank, same statistics
+    n_of = {f: xs[f].numel() for f in fields}
+    nmax = max(n_of.values())
+    ws = cz.Workspace(nmax, dev)
+    cap = cz.max_compressed_bytes(nmax)
+    out = torch.empty(cap, dtype=torch.uint8, device=dev)
+    out_bytes = torch.zeros(1, dtype=torch.int64, device=dev)
+    y = torch.empty(nmax, dtype=torch.float32, device=dev)
+    mm_local = torch.empty(2, dtype=torch.float32, device=dev)
+    mm_all = torch.empty(2 * world, dtype=torch.float32, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    jobs = [(f, r) for f in fields for r in rels]
+    group = torch.distributed.group.WORLD if world > 1 else None
+
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in jobs]
+    acc = {"range": 0.0, "compress": 0.0, "decompress": 0.0}
+    sizes = {}
+
+    def one_step(timed: bool):
+        for j, (f, rel) in enumerate(jobs):
+            x = xs[f]
+            n = n_of[f]
+            flush.zero_()                                   # L2 flush, untimed
+            e = ev[j]
+            e[0].record(stream)
+            cz.check(lib.cuszp_range(x.data_ptr(), n, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
+            if world > 1:
+                czd.allgather_minmax(mm_local, mm_all, group)   # global REL range over NVLink
+                mm, pairs = mm_all, world
+            else:
+                mm, pairs = mm_local, 1
+            e[1].record(stream)
+            cz.check(lib.cuszp_compress_minmax(x.data_ptr(), n, float(rel), mm.data_ptr(), pairs, out.data_ptr(),
+                                               cap, out_bytes.data_ptr(), ws.ptr(), ws.nbytes, sp), "compress")
+            if world > 1:
+                czd.allgather_sizes(out_bytes, group)          # container header offsets
+            e[2].record(stream)
+            cz.check(lib.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.ptr(), ws.nbytes, sp),
+                     "decompress")
+            e[3].record(stream)
+            if timed:
+                torch.cuda.synchronize(dev)
+                acc["range"] += e[0].elapsed_time(e[1])
+                acc["compress"] += e[1].elapsed_time(e[2])
+                acc["decompress"] += e[2].elapsed_time(e[3])
+                sizes[(f, rel)] = int(out_bytes.item())
+
+    for _ in range(max(args.warmup, 3)):
+        one_step(False)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize(dev)
+    clocks = ClockSampler(dev.index)
+    clocks.start()
+    t_wall0 = time.perf_counter()
+    for _ in range(args.steps):
+        one_step(True)
+    torch.cuda.synchronize(dev)
+    t_wall = time.perf_counter() - t_wall0
+    clk = clocks.stop()
+    if world > 1:
+        torch.distributed.barrier()
+
+    # correctness spot check of the last round trip (device-side, bound of DESIGN sec 5)
+    f_last, rel_last = jobs[-1]
+    hdr = cz.read_header(out)
+    assert hdr["status"] == 0 and cz.last_status(ws) == cz.OK
+    xl = xs[f_last]
+    err = (y[: xl.numel()].double() - xl.double()).abs().max().item()
+    ulp_max = float(np.spacing(np.float32(xl.abs().max().item())))
+    assert err <= hdr["eb_abs"] + ulp_max, (err, hdr["eb_abs"])
+
+    t_dev = torch.tensor([acc["range"], acc["compress"], acc["decompress"]], dtype=torch.float64, device=dev)
+    if world > 1:
+        torch.distributed.all_reduce(t_dev, op=torch.distributed.ReduceOp.MAX)
+    t_range, t_comp, t_decomp = (float(v) / 1e3 for v in t_dev.tolist())   # seconds over K steps
+    K = args.steps
+    in_bytes_step = sum(4 * n_of[f] for f, _ in jobs)
+    total_bytes = in_bytes_step * K * world
+    t_step_total = t_range + t_comp + t_decomp
+    S = {k: v for k, v in sizes.items()}
+    cr = {f"{f}@{r:g}": round(4 * n_of[f] / S[(f, r)], 3) for f, r in jobs}
+
+    peak, peak_src = peak_hbm()
+    per_launch = {
+        "range": sum(4 * n_of[f] for f, _ in jobs) / (t_range / K),
+        "compress": sum(4 * n_of[f] + S[(f, r)] for f, r in jobs) / (t_comp / K),
+        "decompress": sum(S[(f, r)] + 4 * n_of[f] for f, r in jobs) / (t_decomp / K),
+    }
+    times = {"range": t_range, "compress": t_comp, "decompress": t_decomp}
+    dom = max(times, key=times.get)
+    achieved = per_launch[dom] / 1e9
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as fh:
+            traffic = json.load(fh).get("dram_bytes_per_launch", {}).get(dom)
+    except Exception:
+        pass
+
+    line = {
+        "metric": "end-to-end compress+decompress GB/s (input fp32), REL, incl. range kernel",
+        "value": total_bytes / t_step_total / 1e9 / K * K,
+        "unit": "GB/s", "n_gpus": world, "steps": K, "warmup": max(args.warmup, 3),
+        "ms_per_step": t_step_total / K * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": args.config, "fields": [f for f in fields if f] or None, "rel": rels,
+                   "n_per_field": n_of[fields[0]], "round_trips_per_step": len(jobs),
+                   "parallelism": f"dp{world}" if world > 1 else "single",
+                   "l2": "flushed (512 MB write, untimed) before every round trip"},
+        "compress_gbs": in_bytes_step * K * world / (t_range + t_comp) / 1e9,
+        "compress_kernel_only_gbs": in_bytes_step * K * world / t_comp / 1e9,
+        "decompress_gbs": in_bytes_step * K * world / t_decomp / 1e9,
+        "cr": cr,
+        "kernels": {k: {"ms_per_step": times[k] / K * 1e3, "algorithmic_gbs": per_launch[k] / 1e9,
+                        "frac_of_peak": per_launch[k] / 1e9 / peak} for k in times},
+        "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
+        "gpu_launches": 3 * len(jobs) * K,
+        "clocks": clk,
+        "wall_s_timed_region": t_wall,
+        "paper_context": PAPER_A100,
+    }
+
+    # ---- e2e through the host-buffer C-ABI calls (pinned memory)
+    if not args.no_e2e:
+        h_in = {f: xs[f].cpu().pin_memory() for f in fields}
+        h_out = torch.empty(cap, dtype=torch.uint8).pin_memory()
+        h_y = torch.empty(nmax, dtype=torch.float32).pin_memory()
+        d_in = torch.empty(nmax, dtype=torch.float32, device=dev)
+        h2d = d2h = 0
+        for i in range(1 + args.steps):
+            if i == 1:
+                torch.cuda.synchronize(dev)
+                if world > 1:
+                    torch.distributed.barrier()
+                t0 = time.perf_counter()
+                h2d = d2h = 0
+            for f, rel in jobs:
+                n = n_of[f]
+                nb = cz.compress_host(h_in[f], rel, "rel", h_out, d_in, out, ws)
+                cz.decompress_host(h_out, nb, h_y[:n], out, y, ws)
+                h2d += 4 * n + nb
+                d2h += 8 + nb + 4 * n
+        t_e2e = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+        if world > 1:
+            torch.distributed.all_reduce(t_e2e, op=torch.distributed.ReduceOp.MAX)
+        line["e2e"] = {"value": in_bytes_step * K * world / float(t_e2e.item()) / 1e9, "unit": "GB/s",
+                       "h2d_bytes_per_step": h2d // K, "d2h_bytes_per_step": d2h // K,
+                       "path": "cuszp_compress_host + cuszp_decompress_host (pinned host buffers, wall clock)"}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(args, args.config, fields, rels)
+    return line
+
+
+def main():
+    args = parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        torch.distributed.init_process_group("nccl", device_id=dev)
+    line = run_ours(args, rank, world, dev)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -16,7 +16,7 @@
  *  - d_ pointers are CUDA device pointers, h_ pointers host pointers.
  *  - The caller owns (allocates, frees) every buffer.  The asynchronous
  *    calls never allocate, never synchronise and are CUDA-Graph capturable.
- *  - Device buffers must be 16-byte aligned (d_in of compress: 4-byte).
+ *  - Device buffers must be 16-byte aligned (d_in of cuszp_range: 4-byte).
  *  - A workspace d_ws of cuszp_workspace_bytes(n) bytes must be ZEROED ONCE
  *    when allocated (e.g. cudaMemset) and may then be reused for any number
  *    of calls with element counts <= n.  Calls sharing a workspace must be

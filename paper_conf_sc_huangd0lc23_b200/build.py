@@ -48,15 +48,20 @@ def needs_build() -> bool:
     return any(os.path.getmtime(d) > t for d in deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, defines: list[str] | None = None,
+          out: str | None = None) -> str:
+    """Compile every csrc/*.cu into one shared library (default: the in-tree
+    libcuszp.so).  ``defines``/``out`` build diagnostic variants elsewhere."""
+    target = out or LIB
+    if out is None and not force and not needs_build():
         return LIB
-    cmd = [nvcc(), *ARCH, *NVCC_FLAGS, "-shared", "-o", LIB + ".tmp", *sources()]
+    cmd = [nvcc(), *ARCH, *NVCC_FLAGS, *[f"-D{d}" for d in (defines or [])], "-shared", "-o", target + ".tmp",
+           *sources()]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     subprocess.run(cmd, check=True)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

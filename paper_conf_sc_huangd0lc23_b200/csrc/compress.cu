@@ -1,48 +1,118 @@
 // compress.cu -- the fused cuSZp compression kernel for sm_100a
 // (paper sec 3.1 / Fig 2 and sec 4).
 //
-// One launch does, per 2048-element tile taken by ticket:
-//   a2 pre-quantisation   r = round(d / 2eb)              (R2)
-//   a3 block Lorenzo      l_j = r_j - r_{j-1}, r_{-1}=0
-//   a4 sign map           ballot(l < 0)                    (R7)
-//   a5 fixed length       F = 32 - clz(redux.max |l|)
-//   a6 CmpL               4 (F + 1) bytes, 0 if F = 0      (Eq 2, R6)
-//   a7 global sync        warp / CTA prefix + decoupled look-back (Eq 3,
-//                         hierarchy of Fig 9)
-//   a8 bit-shuffle        plane k = ballot(bit k of |l|), stored with the
-//                         sign map at the scanned offset   (R9)
-// Layout in the output stream: DESIGN.md sec 4.
+// Persistent, warp-specialised CTA:
+//   warp 0      producer: takes a tile ticket, streams the tile's 16 KB of
+//               fp32 HBM -> shared memory with one 1D TMA bulk copy
+//               (UBLKCP) into a 3-stage mbarrier ring;
+//   warps 2..9  compute: 16 L-blocks each, one lane per element:
+//     a2 pre-quantisation   r = round(d / 2eb)            (R2)
+//     a3 block Lorenzo      l_j = r_j - r_{j-1}, r_{-1}=0
+//     a4 sign map + a8 bit-shuffle: v_j = 2|l_j| + [l_j<0]; a warp bit
+//        transpose of v turns lane k into word k of the block: sign map
+//        (k=0) then plane k-1 (R7, R9).  Two blocks
+//        with F <= 15 share one transpose (bits 0-15 / 16-31).
+//     a5 fixed length       words = bitlen(redux.max v) = F+1 (0: zero block)
+//     a6 CmpL               4 * words bytes                 (Eq 2, R6)
+//     payload words go to a shared-memory staging buffer, F bytes to HBM;
+//     the last compute warp to finish a tile publishes the tile aggregate
+//     (a7, first half of the decoupled look-back) at once;
+//   warps 1..3  writers, one per staging slot: resolve the tile's prefix by
+//               look-back (a7, Eq 3) and copy the staged words to
+//               their global offsets, while the compute warps already work on
+//               the next tiles (three look-backs in flight per CTA).
 #include "internal.cuh"
 
 namespace cuszp {
 
 namespace {
 
-// Quantise one element with the R2 op sequence (explicit RN intrinsics:
-// never contracted, identical to the oracle's separately rounded ops).
-__device__ __forceinline__ int quantize(float x, float eb, float two_eb, float recip, bool& ok) {
+#ifndef CUSZP_C_STAGES
+#define CUSZP_C_STAGES 3
+#endif
+#ifndef CUSZP_C_STAGING
+#define CUSZP_C_STAGING 5
+#endif
+#ifndef CUSZP_C_MINBLOCKS
+#define CUSZP_C_MINBLOCKS 2
+#endif
+constexpr int kStages = CUSZP_C_STAGES;     // input ring depth
+constexpr int kStaging = CUSZP_C_STAGING;   // payload staging buffers = writer warps
+constexpr int kWarpWords = kBPW * kMaxBlockWords;   // 400 words per warp region
+constexpr int kFirstCompute = 1 + kStaging;         // warp index of compute warp 0
+constexpr int kCThreads = (kFirstCompute + kComputeWarps) * 32;
+
+struct CompressSmem {
+  float in[kStages][kTileElems];                              // 48 KB
+  uint32_t words[kStaging][kComputeWarps][kWarpWords];        // 25.6 KB
+  uint32_t warp_words[kStaging][kComputeWarps];
+  uint32_t in_tile[kStages];
+  uint32_t st_tile[kStaging];
+  uint32_t st_agg[kStaging];
+  uint32_t st_done[kStaging];      // compute warps finished with the slot's tile
+  uint64_t full[kStages], empty[kStages], staged[kStaging], freed[kStaging];
+};
+
+// R2 op sequence with explicit RN intrinsics (never contracted); rint via the
+// 1.5*2^23 magic constant, exact for |v| < 2^22 (the R5 guard).  Returns the
+// quantisation integer r BIASED by the magic's bit pattern (r + 0x4B400000),
+// which the Lorenzo step removes for free.
+//
+// Fast path: r0 = rint(d * recip).  It differs from round(d / 2eb) only when
+// the exact residual |d - r0*2eb| exceeds eb (d/2eb within an ulp of a half
+// integer), and NaN/Inf give a NaN residual: both set `rare`, and the block
+// is then redone with the full correction (quantize_exact) -- same result as
+// the oracle's sequence in every case, at 6 instructions per element.
+__device__ __forceinline__ uint32_t quantize_fast(float x, float eb, float two_eb, float recip, float& vmax,
+                                                  bool& rare) {
   const float v = __fmul_rn(x, recip);
-  ok = fabsf(v) < kGuard;                               // NaN / Inf / overflow -> false (R5)
-  const float t = __fadd_rn(v, kRoundMagic);           // = 1.5*2^23 + rint(v), |v| < 2^22
-  const float r0 = __fsub_rn(t, kRoundMagic);          // rint(v), exact
-  const float res = __fmaf_rn(-r0, two_eb, x);         // d - r0*2eb, exact (R2)
-  int r = int(__float_as_uint(t) - kRoundMagicBits);   // rint(v) as an integer
-  r += int(res > eb) - int(res < -eb);
+  vmax = fmaxf(vmax, fabsf(v));                    // R5 guard (|v| >= 2^22, Inf); NaN -> `rare`
+  const float t = __fadd_rn(v, kRoundMagic);
+  const float r0 = __fsub_rn(t, kRoundMagic);
+  const float res = __fmaf_rn(-r0, two_eb, x);     // exact residual (R2)
+  rare = !(fabsf(res) <= eb);
+  return __float_as_uint(t);
+}
+
+__device__ __forceinline__ uint32_t quantize_exact(float x, float eb, float two_eb, float recip, float& vmax) {
+  const float v = __fmul_rn(x, recip);
+  if (!(fabsf(v) < kGuard)) vmax = __int_as_float(0x7f800000);   // NaN too
+  const float t = __fadd_rn(v, kRoundMagic);
+  const float r0 = __fsub_rn(t, kRoundMagic);
+  const float res = __fmaf_rn(-r0, two_eb, x);
+  uint32_t r = __float_as_uint(t);
+  r += uint32_t(int(res > eb) - int(res < -eb));
   return r;
+}
+
+// lane j holds the biased r_j of one block -> v_j = 2|l_j| + sign_j with the
+// block Lorenzo l_j = r_j - r_{j-1}, r_{-1} = 0
+__device__ __forceinline__ uint32_t lorenzo_pack(uint32_t rb, int lane) {
+  uint32_t prev = __shfl_up_sync(kFull, rb, 1);
+  prev = lane ? prev : kRoundMagicBits;
+  const int l = int(rb - prev);
+  const uint32_t a = uint32_t(l < 0 ? -l : l);
+  return (a << 1) | (uint32_t(l) >> 31);
+}
+
+// words of a block = bit length of max v = F + 1 (0 for a zero block)
+__device__ __forceinline__ uint32_t word_count(uint32_t v) {
+  const uint32_t m = __reduce_max_sync(kFull, v);
+  uint32_t b;
+  asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(m));   // 0xffffffff for m = 0
+  return b + 1;
 }
 
 }  // namespace
 
-__global__ void __launch_bounds__(kThreads) compress_kernel(CompressArgs a) {
-  __shared__ uint32_t s_tile;
-  __shared__ uint32_t s_warp_words[kWarps];
-  __shared__ uint64_t s_warp_base[kWarps];
-
+__global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(CompressArgs a) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const uint32_t epoch = running_epoch(a.ws);
 
-  // ---- resolve eb_abs (Eq 1): ABS -> delta; REL -> lambda * (max - min) over the pairs
+  // ---- eb_abs (Eq 1): ABS -> delta; REL -> lambda * (max - min) over the (min,max) pairs
   float eb = a.eb_in;
   if (a.mode == CUSZP_REL) {
     float mn = a.minmax[0], mx = a.minmax[1];
@@ -53,108 +123,200 @@ __global__ void __launch_bounds__(kThreads) compress_kernel(CompressArgs a) {
       if (lo < mn) mn = lo;
       if (hi > mx) mx = hi;
     }
-    eb = __fmul_rn(a.eb_in, __fsub_rn(mx, mn));         // R3
+    eb = __fmul_rn(a.eb_in, __fsub_rn(mx, mn));   // R3
     if (nan) eb = __int_as_float(0x7fc00000);
   }
   const float two_eb = __fadd_rn(eb, eb);
   const bool eb_ok = (eb >= kFltMin) && isfinite(two_eb) && a.n > 0;   // R5
   const float recip = __fdiv_rn(1.0f, two_eb);
-
-  uint32_t bad = (a.n > 0 && !eb_ok) ? kBadRange : 0u;
+  float vmax = 0.0f;        // max over this thread's elements of |d / 2eb| (R5 guard)
   const uint64_t p0 = kHdr + align16(a.nb);
   uint32_t* payload = reinterpret_cast<uint32_t*>(a.out + p0);
 
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kComputeWarps); }
+    for (int b = 0; b < kStaging; ++b) {
+      mbar_init(&sm.staged[b], 1);
+      mbar_init(&sm.freed[b], 1);
+      sm.st_done[b] = 0;
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+
   if (eb_ok) {
-    while (true) {
-      if (threadIdx.x == 0) s_tile = atomicAdd(&a.ws->ticket, 1u);
-      __syncthreads();
-      const uint32_t t = s_tile;
-      if (t >= a.num_tiles) break;
-
-      const uint64_t blk0 = uint64_t(t) * kTileBlocks + uint64_t(warp) * kBPW;
-
-      // -- load: lane j <- element j of each of the warp's 8 blocks (coalesced 128 B rows)
-      float x[kBPW];
-#pragma unroll
-      for (int b = 0; b < kBPW; ++b) {
-        const uint64_t idx = (blk0 + b) * kL + lane;
-        x[b] = idx < a.n ? ld_stream_f32(a.in + idx) : 0.0f;    // virtual zero pad (R8)
-      }
-
-      // -- per block: quantise, predict, encode (all in registers)
-      uint32_t word[kBPW];   // lane 0: sign map, lane k+1: plane k
-      uint32_t F[kBPW];      // warp-uniform
-#pragma unroll
-      for (int b = 0; b < kBPW; ++b) {
-        bool ok;
-        const int r = quantize(x[b], eb, two_eb, recip, ok);
-        if (!ok && (blk0 + b) * kL + lane < a.n) bad |= kBadRange;
-        const int prev = __shfl_up_sync(kFull, r, 1);
-        const int l = (lane == 0) ? r : r - prev;
-        const uint32_t sign = __ballot_sync(kFull, l < 0);
-        const uint32_t mag = uint32_t(l < 0 ? -l : l);
-        const uint32_t m = __reduce_max_sync(kFull, mag);
-        const uint32_t f = 32u - __clz(m);
-        uint32_t w = sign;
-        for (uint32_t k = 0; k < f; ++k) {
-          const uint32_t plane = __ballot_sync(kFull, (mag >> k) & 1u);
-          if (lane == int(k) + 1) w = plane;
+    if (warp == 0) {
+      // ------------------------------------------------------------ producer
+      if (lane == 0) {
+        uint32_t next = atomicAdd(&a.ws->ticket, 1u);   // tickets are prefetched one ahead
+        for (uint32_t i = 0;; ++i) {
+          const int s = int(i % kStages);
+          mbar_wait(&sm.empty[s], ((i / kStages) & 1u) ^ 1u);
+          const uint32_t t = next;
+          if (t >= a.num_tiles) {
+            sm.in_tile[s] = kSentinel;
+            mbar_arrive(&sm.full[s]);
+            break;
+          }
+          next = atomicAdd(&a.ws->ticket, 1u);
+          trace_put(a.trace, t, 0, global_ns());
+          sm.in_tile[s] = t;
+          const uint64_t e0 = uint64_t(t) * kTileElems;
+          const uint64_t ne = min(uint64_t(kTileElems), a.n - e0);
+          const uint32_t bytes = uint32_t(ne * 4);
+          const uint32_t tma_bytes = bytes & ~15u;
+          for (uint32_t k = tma_bytes / 4; k < ne; ++k) sm.in[s][k] = a.in[e0 + k];   // <= 3 tail floats
+          mbar_arrive_expect_tx(&sm.full[s], tma_bytes);
+          if (tma_bytes) tma_load_1d(sm.in[s], a.in + e0, tma_bytes, &sm.full[s]);
         }
-        word[b] = w;
-        F[b] = f;
       }
-
-      // -- hierarchical scan (Fig 9): thread/warp level is a serial sum of the warp's 8 blocks
-      uint32_t pre[kBPW];
-      uint32_t wsum = 0;
-#pragma unroll
-      for (int b = 0; b < kBPW; ++b) {
-        pre[b] = wsum;
-        wsum += F[b] ? F[b] + 1u : 0u;
-      }
-      if (lane == 0) s_warp_words[warp] = wsum;
-      __syncthreads();
-      if (warp == 0) {
-        const uint32_t v = lane < kWarps ? s_warp_words[lane] : 0u;
+    } else if (warp < kFirstCompute) {
+      // ------------------------------------------- writers (one per staging slot)
+      const int b = warp - 1;
+      for (uint32_t j = 0;; ++j) {
+        mbar_wait(&sm.staged[b], j & 1u);
+        const uint32_t t = sm.st_tile[b];
+        if (t == kSentinel) break;
+        const uint32_t agg = sm.st_agg[b];
+        const uint32_t v = lane < kComputeWarps ? sm.warp_words[b][lane] : 0u;
         uint32_t incl = v;
 #pragma unroll
-        for (int o = 1; o < kWarps; o <<= 1) {
+        for (int o = 1; o < kComputeWarps; o <<= 1) {
           const uint32_t y = __shfl_up_sync(kFull, incl, o);
           if (lane >= o) incl += y;
         }
-        const uint32_t agg = __shfl_sync(kFull, incl, kWarps - 1);
-        const uint64_t excl = tile_lookback(a.status, t, agg, epoch);   // global level
-        if (lane < kWarps) s_warp_base[lane] = excl + incl - v;
+        uint32_t nw = 0, ns = 0;
+        const uint64_t t_lb = a.trace ? global_ns() : 0;
+        const uint64_t excl = resolve_prefix(a.status, t, agg, epoch, &nw, &ns);
+        if (lane == 0 && a.trace) {
+          trace_put(a.trace, t, 3, t_lb);
+          trace_put(a.trace, t, 4, global_ns());
+          trace_put(a.trace, t, 5, nw);
+          trace_put(a.trace, t, 6, ns);
+          uint32_t smid;
+          asm("mov.u32 %0, %smid;" : "=r"(smid));
+          trace_put(a.trace, t, 7, (uint64_t(smid) << 32) | blockIdx.x);
+        }
+        // copy every compute warp's staged words to [excl + warp offset ...)
+#pragma unroll 1
+        for (int w = 0; w < kComputeWarps; ++w) {
+          const uint32_t cnt = __shfl_sync(kFull, v, w);
+          const uint32_t off = __shfl_sync(kFull, incl - v, w);
+          uint32_t* dst = payload + excl + off;
+          const uint32_t* src = sm.words[b][w];
+          for (uint32_t k = lane; k < cnt; k += 32) dst[k] = src[k];
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.freed[b]);
       }
-      __syncthreads();
-      const uint64_t base = s_warp_base[warp];
-
-      // -- fixed-length bytes (Fig 12 part 1): 8 blocks -> two u32 stores
-      if (lane < 2 && blk0 + 4 * lane < align16(a.nb)) {
-        const uint32_t lo = F[0] | (F[1] << 8) | (F[2] << 16) | (F[3] << 24);
-        const uint32_t hi = F[4] | (F[5] << 8) | (F[6] << 16) | (F[7] << 24);
-        *reinterpret_cast<uint32_t*>(a.out + kHdr + blk0 + 4 * lane) = lane ? hi : lo;
-      }
-      // -- shuffled bytes at the synchronised offsets (Fig 12 part 2)
+    } else {
+      // ------------------------------------------------------------ compute
+      const int w = warp - kFirstCompute;
+      const Xpose xpose(lane);
+      for (uint32_t i = 0;; ++i) {
+        const int s = int(i % kStages);
+        const int b = int(i % kStaging);
+        mbar_wait(&sm.full[s], (i / kStages) & 1u);
+        const uint32_t t = sm.in_tile[s];
+        if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());   // data landed
+        mbar_wait(&sm.freed[b], ((i / kStaging) & 1u) ^ 1u);   // staging slot b written out
+        if (t == kSentinel) {
+          // every writer must see the sentinel: fill all slots in order
+          if (w == 0 && lane == 0) {
+            for (int k = 0; k < kStaging; ++k) {
+              const int bb = int((i + k) % kStaging);
+              if (k > 0) mbar_wait(&sm.freed[bb], (((i + k) / kStaging) & 1u) ^ 1u);
+              sm.st_tile[bb] = kSentinel;
+              mbar_arrive(&sm.staged[bb]);
+            }
+          }
+          break;
+        }
+        const bool last = (t == a.num_tiles - 1);
+        const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;   // first element of the warp
+        const float* src = &sm.in[s][w * kBPW * 32];
+        uint32_t* stage = sm.words[b][w];
+        uint32_t cursor = 0;
+        uint32_t fpack[4] = {0, 0, 0, 0};
 #pragma unroll
-      for (int b = 0; b < kBPW; ++b) {
-        if (F[b] != 0 && uint32_t(lane) <= F[b]) payload[base + pre[b] + lane] = word[b];
+        for (int p = 0; p < kBPW / 2; ++p) {
+          float xa = src[(2 * p) * 32 + lane];
+          float xb = src[(2 * p + 1) * 32 + lane];
+          if (last) {
+            if (g0 + (2 * p) * 32 + lane >= a.n) xa = 0.0f;         // virtual zero pad (R8)
+            if (g0 + (2 * p + 1) * 32 + lane >= a.n) xb = 0.0f;
+          }
+          bool rare_a, rare_b;
+          uint32_t ra = quantize_fast(xa, eb, two_eb, recip, vmax, rare_a);
+          uint32_t rb = quantize_fast(xb, eb, two_eb, recip, vmax, rare_b);
+          if (__any_sync(kFull, rare_a || rare_b)) {
+            ra = quantize_exact(xa, eb, two_eb, recip, vmax);
+            rb = quantize_exact(xb, eb, two_eb, recip, vmax);
+          }
+          const uint32_t va = lorenzo_pack(ra, lane);
+          const uint32_t vb = lorenzo_pack(rb, lane);
+          const uint32_t wa = word_count(va);
+          const uint32_t wb = word_count(vb);
+          const uint32_t oa = cursor, ob = cursor + wa;
+          cursor = ob + wb;
+          if (wa <= 16 && wb <= 16) {
+            const uint32_t tw = xpose(va | (vb << 16));
+            const bool hi = lane >= 16;
+            const uint32_t k = lane & 15;
+            if (k < (hi ? wb : wa)) stage[(hi ? ob : oa) + k] = tw;
+          } else {
+            const uint32_t ta = xpose(va);
+            if (uint32_t(lane) < wa) stage[oa + lane] = ta;
+            const uint32_t tb = xpose(vb);
+            if (uint32_t(lane) < wb) stage[ob + lane] = tb;
+          }
+          const uint32_t fa = wa ? wa - 1 : 0, fb = wb ? wb - 1 : 0;
+          const uint32_t f2 = fa | (fb << 8);
+          fpack[p >> 1] |= f2 << ((p & 1) * 16);
+        }
+        // F bytes of the warp's 16 blocks (Fig 12 part 1): one 16-byte store
+        const uint64_t blk0 = uint64_t(t) * kTileBlocks + uint64_t(w) * kBPW;
+        if (lane == 0 && blk0 < a.nb)
+          *reinterpret_cast<uint4*>(a.out + kHdr + blk0) = make_uint4(fpack[0], fpack[1], fpack[2], fpack[3]);
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(&sm.empty[s]);                       // input stage consumed
+          sm.warp_words[b][w] = cursor;
+          __threadfence_block();
+          if (atomicAdd(&sm.st_done[b], 1u) == kComputeWarps - 1) {
+            // last warp of the tile: aggregate -> publish at once (look-back, part 1)
+            __threadfence_block();
+            uint32_t agg = 0;
+#pragma unroll
+            for (int k = 0; k < kComputeWarps; ++k) agg += *reinterpret_cast<volatile uint32_t*>(&sm.warp_words[b][k]);
+            publish_aggregate(a.status, t, agg, epoch);
+            trace_put(a.trace, t, 2, global_ns());
+            sm.st_tile[b] = t;
+            sm.st_agg[b] = agg;
+            sm.st_done[b] = 0;
+            mbar_arrive(&sm.staged[b]);
+          }
+        }
       }
     }
   }
 
-  if (cta_finish(a.ws, bad)) {
+  // R5 guard: some |d / 2eb| >= 2^22 (NaN and Inf have larger bit patterns)
+  uint32_t flag = 0;
+  if (!eb_ok) flag = (a.n > 0) ? kBadRange : 0u;
+  else if (!(vmax < kGuard)) flag = kBadRange;
+
+  if (cta_finish(a.ws, flag)) {
     uint32_t final_status = CUSZP_OK;
-    uint64_t total_words = 0;
     if (threadIdx.x == 0) {
       const uint32_t acc = *reinterpret_cast<volatile uint32_t*>(&a.ws->status_accum);
       if (acc & kBadRange) final_status = CUSZP_ERANGE;
+      uint64_t total_words = 0;
       if (final_status == CUSZP_OK && a.num_tiles > 0)
         total_words = ld_relaxed_u64(a.status + a.num_tiles - 1) & kValueMask;
       const uint64_t payload_bytes = final_status == CUSZP_OK ? total_words * 4 : 0;
-      // header (R10)
-      uint8_t* h = a.out;
-      *reinterpret_cast<uint32_t*>(h) = 0x505A5343u;   // "CSZP"
+      uint8_t* h = a.out;                                   // header (R10)
+      *reinterpret_cast<uint32_t*>(h) = 0x505A5343u;        // "CSZP"
       h[4] = CUSZP_VERSION;
       h[5] = uint8_t(a.mode);
       h[6] = uint8_t(final_status);
@@ -163,11 +325,13 @@ __global__ void __launch_bounds__(kThreads) compress_kernel(CompressArgs a) {
       *reinterpret_cast<float*>(h + 16) = a.n > 0 ? eb : (a.mode == CUSZP_REL ? 0.0f : a.eb_in);
       *reinterpret_cast<float*>(h + 20) = a.eb_in;
       *reinterpret_cast<uint64_t*>(h + 24) = payload_bytes;
-      if (a.out_bytes)
-        *a.out_bytes = (a.n == 0) ? uint64_t(kHdr) : p0 + payload_bytes;
+      if (a.out_bytes) *a.out_bytes = (a.n == 0) ? uint64_t(kHdr) : p0 + payload_bytes;
     }
     finish_call(a.ws, a.status, a.status_cap, epoch, final_status);
   }
 }
+
+size_t compress_smem_bytes() { return sizeof(CompressSmem); }
+int compress_threads() { return kCThreads; }
 
 }  // namespace cuszp

@@ -19,7 +19,8 @@ struct DeviceInfo {
   int occ_compress = 0, occ_decompress = 0, occ_range = 0;
 };
 
-// Per-device launch geometry, computed once (occupancy of each kernel).
+// Per-device launch geometry, computed once: persistent grids of
+// (SM count x resident CTAs per SM) for the two scan kernels.
 int device_info(DeviceInfo* out) {
   static std::mutex mu;
   static DeviceInfo cache[64];
@@ -29,9 +30,14 @@ int device_info(DeviceInfo* out) {
   std::lock_guard<std::mutex> lock(mu);
   if (!have[dev]) {
     DeviceInfo d;
-    if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return CUSZP_ECUDA;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_compress, compress_kernel, kThreads, 0) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_decompress, decompress_kernel, kThreads, 0) != cudaSuccess ||
+    const int cs = int(compress_smem_bytes()), ds = int(decompress_smem_bytes());
+    if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
+        cudaFuncSetAttribute(compress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
+        cudaFuncSetAttribute(decompress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess)
+      return CUSZP_ECUDA;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_compress, compress_kernel, compress_threads(), cs) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_decompress, decompress_kernel, decompress_threads(), ds) !=
+            cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess)
       return CUSZP_ECUDA;
     cache[dev] = d;
@@ -46,6 +52,10 @@ bool eb_is_normal(float eb) {
   const float two = eb + eb;
   return two - two == 0.0f;   // finite
 }
+
+// Diagnostics: a device buffer of 8 u64 per tile filled by the next launches
+// (tools/trace_scan.py).  Not part of include/cuszp.h; nullptr in production.
+uint64_t* g_trace = nullptr;
 
 uint32_t status_capacity(size_t ws_bytes) {
   const uint64_t c = (ws_bytes - kWsCtrlBytes) / 8;
@@ -73,10 +83,11 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   a.ws = static_cast<WsCtrl*>(d_ws);
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
+  a.trace = g_trace;
   uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_compress > 0 ? di.occ_compress : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  compress_kernel<<<unsigned(grid), kThreads, 0, stream>>>(a);
+  compress_kernel<<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
   return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
@@ -119,7 +130,7 @@ int cuszp_range(const float* d_in, size_t n, float* d_minmax, void* d_ws, size_t
 int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out, size_t out_capacity,
                    unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes, void* stream) {
   if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr) return CUSZP_EINVAL;
-  if ((reinterpret_cast<uintptr_t>(d_in) & 3u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
+  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -149,7 +160,7 @@ int cuszp_compress_minmax(const float* d_in, size_t n, float lambda, const float
   if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || d_minmax == nullptr ||
       n_pairs <= 0)
     return CUSZP_EINVAL;
-  if ((reinterpret_cast<uintptr_t>(d_in) & 3u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
+  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
   if (!(lambda > 0.0f) || !(lambda - lambda == 0.0f)) return CUSZP_EINVAL;
@@ -160,7 +171,7 @@ int cuszp_compress_minmax(const float* d_in, size_t n, float lambda, const float
 int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n, void* d_ws, size_t ws_bytes,
                      void* stream) {
   if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr) return CUSZP_EINVAL;
-  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 3u) ||
+  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
   if (ws_bytes < cuszp_workspace_bytes(n)) return CUSZP_ENOSPACE;
@@ -176,10 +187,12 @@ int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n, 
   a.ws = static_cast<WsCtrl*>(d_ws);
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
+  a.trace = g_trace;
   uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_decompress > 0 ? di.occ_decompress : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  decompress_kernel<<<unsigned(grid), kThreads, 0, static_cast<cudaStream_t>(stream)>>>(a);
+  decompress_kernel<<<unsigned(grid), decompress_threads(), decompress_smem_bytes(),
+                      static_cast<cudaStream_t>(stream)>>>(a);
   return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
@@ -259,5 +272,8 @@ const char* cuszp_status_string(int status) {
 }
 
 int cuszp_version(void) { return CUSZP_VERSION * 100 + 1; }
+
+// diagnostics only (not declared in include/cuszp.h)
+void cuszp_debug_set_trace(void* d_trace) { g_trace = static_cast<uint64_t*>(d_trace); }
 
 }  // extern "C"

@@ -1,13 +1,16 @@
 // internal.cuh -- device-side definitions shared by the three kernels of the
 // B200-native cuSZp path (sm_100a).  Nothing here is shared with oracle/.
 //
-// Design: persistent CTAs take TILES of 64 L-blocks
-// (8 warps x 8 blocks) by atomic ticket; within a warp one lane owns one
-// element of a 32-element block (lane j <-> element j), so the paper's
-// per-block steps become warp primitives: Lorenzo = shfl_up, sign map and
-// bit planes = ballot, max = redux.max, F = 32 - clz.  Tiles are placed by
-// a decoupled look-back scan (the paper's chained scan) whose
-// status words are epoch-tagged so no memset is needed between calls.
+// Design: persistent, warp-specialised CTAs take TILES of
+// 128 L-blocks (4096 elements, 16 KB of fp32) by atomic ticket.  A producer
+// warp streams tiles HBM -> shared memory with 1D TMA bulk copies into an
+// mbarrier ring; compute warps own 16 blocks each with one lane per element
+// (lane j <-> element j), so the paper's per-block steps become warp
+// primitives (Lorenzo = shfl_up, max = redux.max, F = clz, bit-shuffle =
+// a 15-instruction warp bit-transpose that handles two blocks at once); a
+// scan warp places each tile with a decoupled look-back (the paper's
+// chained scan) over epoch-tagged status words, so no memset is
+// needed between calls and the look-back latency overlaps the next tile.
 #pragma once
 
 #include <cstdint>
@@ -27,10 +30,12 @@ constexpr float kFltMin = 1.17549435e-38f;
 constexpr uint32_t kFull = 0xffffffffu;
 
 // Tile geometry (both scan kernels).
-constexpr int kWarps = 8;                     // warps per CTA
-constexpr int kThreads = kWarps * 32;
-constexpr int kBPW = 8;                       // L-blocks per warp per tile
-constexpr int kTileBlocks = kWarps * kBPW;    // 64 blocks = 2048 elements per tile
+constexpr int kComputeWarps = 8;
+constexpr int kBPW = 16;                                  // L-blocks per compute warp per tile
+constexpr int kTileBlocks = kComputeWarps * kBPW;         // 128 blocks = 4096 elements
+constexpr int kTileElems = kTileBlocks * 32;
+constexpr int kMaxBlockWords = kMaxF + 1;                 // sign map + 24 planes
+constexpr uint32_t kSentinel = 0xffffffffu;
 
 // ---------------------------------------------------------------- workspace
 struct WsCtrl {
@@ -84,6 +89,114 @@ __device__ __forceinline__ float4 ld_stream_f32x4(const float4* p) {
   return v;
 }
 
+// ------------------------------------------------------- mbarrier / TMA bulk
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.release.cta.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+// Blocks until the phase with the given parity has completed.  try_wait
+// suspends the warp in hardware (it stops competing for issue slots) until
+// the phase completes or the suspend-time hint (ns) expires.
+#ifndef CUSZP_SUSPEND_NS
+#define CUSZP_SUSPEND_NS 100000
+#endif
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
+      " @!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity), "n"(CUSZP_SUSPEND_NS)
+      : "memory");
+}
+// One suspending try (true once the phase has completed).
+__device__ __forceinline__ bool mbar_try(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n"
+      " selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity), "n"(CUSZP_SUSPEND_NS)
+      : "memory");
+  return ok != 0;
+}
+// Non-blocking probe: has the phase with the given parity completed?
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      " mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      " selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// 1D TMA bulk copy global -> shared (UBLKCP); 16-byte aligned, size % 16 == 0.
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// ------------------------------------------------------------- bit transpose
+// 32x32 bit-matrix transpose across a warp (lane r holds row r; afterwards
+// lane k holds the word whose bit j is bit k of the old row j).  Five
+// butterfly stages, each ONE shuffle + ONE rotate + ONE 3-input LOP: the
+// rotate amount and keep-mask are per-lane constants, which makes both
+// halves of every exchange execute the same instruction (no divergence).
+// This is the paper's Block Bit-shuffle done for 32 elements
+// at once, and -- being an involution up to layout -- also its inverse.
+struct Xpose {
+  uint32_t amt[5];
+  uint32_t keep[5];
+  __device__ __forceinline__ explicit Xpose(int lane) {
+    const uint32_t m[5] = {0x0000FFFFu, 0x00FF00FFu, 0x0F0F0F0Fu, 0x33333333u, 0x55555555u};
+#pragma unroll
+    for (int s = 0; s < 5; ++s) {
+      const int j = 16 >> s;
+      const bool low = (lane & j) == 0;
+      amt[s] = low ? uint32_t(j) : uint32_t(32 - j);
+      keep[s] = low ? m[s] : ~m[s];
+    }
+  }
+  __device__ __forceinline__ uint32_t operator()(uint32_t x) const {
+#pragma unroll
+    for (int s = 0; s < 5; ++s) {
+      const uint32_t t = __shfl_xor_sync(0xffffffffu, x, 16 >> s);
+      const uint32_t r = __funnelshift_l(t, t, amt[s]);   // rotate left
+      x = (x & keep[s]) | (r & ~keep[s]);
+    }
+    return x;
+  }
+};
+
+// ------------------------------------------------------------- diagnostics
+__device__ __forceinline__ uint64_t global_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+// trace[8 t + slot] = value (only when a trace buffer was installed)
+__device__ __forceinline__ void trace_put(uint64_t* trace, uint32_t t, int slot, uint64_t v) {
+  if (trace) trace[8ull * t + slot] = v;
+}
+
 // ------------------------------------------------------------- warp helpers
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
@@ -99,39 +212,92 @@ __device__ __forceinline__ uint32_t running_epoch(const WsCtrl* ws) {
 }
 
 // Decoupled look-back (single pass; the paper's "chained-scan
-// parallelization", refs [22],[37]).  Called by all 32 lanes of
-// ONE warp of the CTA owning tile t with that tile's aggregate `agg` (in
-// 4-byte words).  Publishes the aggregate, walks predecessors 32 at a
-// time, publishes the inclusive prefix and returns the exclusive one.
-__device__ __forceinline__ uint64_t tile_lookback(uint64_t* status, uint32_t t, uint64_t agg,
+// parallelization", refs [22],[37]), split in two so that the
+// aggregate is published the moment it is known and the (latency-bound)
+// prefix resolution runs on a warp of its own.
+//
+// publish_aggregate: one thread; tile 0's aggregate is already its prefix.
+__device__ __forceinline__ void publish_aggregate(uint64_t* status, uint32_t t, uint64_t agg,
                                                   uint32_t epoch) {
+  const uint64_t tag = uint64_t(epoch) << kEpochShift;
+  st_relaxed_u64(status + t, tag | (t == 0 ? kPrefixFlag : 0ull) | agg);
+}
+
+// resolve_prefix: all 32 lanes of one warp.  Inspects predecessors in
+// windows of 32*K (K status words per lane, loads in flight together), stops
+// at the nearest inclusive prefix, publishes tile t's inclusive prefix and
+// returns its exclusive prefix (in 4-byte words).  Polling backs off
+// exponentially: thousands of warps may be waiting at once, and their loads
+// share the L2 with the data streams.
+#ifndef CUSZP_LB_K
+#define CUSZP_LB_K 1
+#endif
+#ifndef CUSZP_LB_BACKOFF_MIN
+#define CUSZP_LB_BACKOFF_MIN 64
+#endif
+#ifndef CUSZP_LB_BACKOFF_MAX
+#define CUSZP_LB_BACKOFF_MAX 1024
+#endif
+__device__ __forceinline__ uint64_t resolve_prefix(uint64_t* status, uint32_t t, uint64_t agg,
+                                                   uint32_t epoch, uint32_t* n_windows = nullptr,
+                                                   uint32_t* n_spins = nullptr) {
+  if (t == 0) return 0;
+  constexpr int K = CUSZP_LB_K;
+  uint32_t windows = 0, spins = 0;
   const int lane = threadIdx.x & 31;
   const uint64_t tag = uint64_t(epoch) << kEpochShift;
-  if (t == 0) {
-    if (lane == 0) st_relaxed_u64(status, tag | kPrefixFlag | agg);
-    return 0;
-  }
-  if (lane == 0) st_relaxed_u64(status + t, tag | agg);
   uint64_t excl = 0;
-  int64_t base = int64_t(t) - 1;
+  int64_t top = int64_t(t) - 1;          // nearest predecessor not yet summed
+  uint32_t backoff = CUSZP_LB_BACKOFF_MIN;
   while (true) {
-    const int64_t idx = base - lane;
-    uint64_t w;
-    int spins = 0;
+    uint64_t w[K];
     while (true) {
-      w = (idx >= 0) ? ld_relaxed_u64(status + idx) : (tag | kPrefixFlag);
-      const bool ready = (w >> kEpochShift) == epoch;
+      bool ready = true;
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const int64_t idx = top - K * lane - k;   // distance K*lane + k from `top`
+        w[k] = (idx >= 0) ? ld_relaxed_u64(status + idx) : (tag | kPrefixFlag);
+        ready &= (w[k] >> kEpochShift) == epoch;
+      }
       if (__all_sync(kFull, ready)) break;
-      if (++spins > 4) __nanosleep(64);
+      ++spins;
+      __nanosleep(backoff);
+      backoff = min(backoff * 2u, uint32_t(CUSZP_LB_BACKOFF_MAX));
     }
-    const uint32_t pmask = __ballot_sync(kFull, (w & kPrefixFlag) != 0);
+    ++windows;
+    // per lane: aggregates up to and including its first prefix (k = distance order)
+    uint64_t part = 0;
+    bool has_p = false;
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      if (!has_p) {
+        part += w[k] & kValueMask;
+        has_p = (w[k] & kPrefixFlag) != 0;
+      }
+    }
+    const uint32_t pmask = __ballot_sync(kFull, has_p);
     const int stop = pmask ? (__ffs(pmask) - 1) : 31;
-    excl += warp_sum_u64(lane <= stop ? (w & kValueMask) : 0);
+    excl += warp_sum_u64(lane <= stop ? part : 0ull);
     if (pmask) break;
-    base -= 32;
+    top -= 32 * K;
   }
   if (lane == 0) st_relaxed_u64(status + t, tag | kPrefixFlag | (excl + agg));
+  if (n_windows) *n_windows = windows;
+  if (n_spins) *n_spins = spins;
   return excl;
+}
+
+// Inclusive scan step with the hardware's in-range predicate (SHFL + @p IADD,
+// no select): x += x[lane - o] when that lane lies in the same segment.
+// seg_c = (32 - segment width) << 8.
+__device__ __forceinline__ int scan_step_up(int x, int o, int seg_c) {
+  asm volatile(
+      "{\n .reg .pred p;\n .reg .b32 t;\n"
+      " shfl.sync.up.b32 t|p, %0, %1, %2, 0xffffffff;\n"
+      " @p add.s32 %0, %0, t;\n}"
+      : "+r"(x)
+      : "r"(o), "r"(seg_c));
+  return x;
 }
 
 // End-of-kernel bookkeeping: accumulate this CTA's status bits, count the
@@ -188,6 +354,7 @@ struct CompressArgs {
   WsCtrl* ws;
   uint64_t* status;
   uint32_t status_cap;
+  uint64_t* trace;           // diagnostics only (nullptr): 8 u64 per tile, see tools/trace_scan.py
 };
 
 struct DecompressArgs {
@@ -200,6 +367,7 @@ struct DecompressArgs {
   WsCtrl* ws;
   uint64_t* status;
   uint32_t status_cap;
+  uint64_t* trace;
 };
 
 struct RangeArgs {
@@ -212,5 +380,9 @@ struct RangeArgs {
 __global__ void compress_kernel(CompressArgs a);
 __global__ void decompress_kernel(DecompressArgs a);
 __global__ void range_kernel(RangeArgs a);
+size_t compress_smem_bytes();
+int compress_threads();
+size_t decompress_smem_bytes();
+int decompress_threads();
 
 }  // namespace cuszp
