@@ -15,12 +15,14 @@
 //     a5 fixed length       words = bitlen(redux.max v) = F+1 (0: zero block)
 //     a6 CmpL               4 * words bytes                 (Eq 2, R6)
 //     payload words go to a shared-memory staging buffer, F bytes to HBM;
+//     each compute warp appends its words to its own shared-memory ring;
 //     the last compute warp to finish a tile publishes the tile aggregate
 //     (a7, first half of the decoupled look-back) at once;
-//   warps 1..3  writers, one per staging slot: resolve the tile's prefix by
-//               look-back (a7, Eq 3) and copy the staged words to
-//               their global offsets, while the compute warps already work on
-//               the next tiles (three look-backs in flight per CTA).
+//   warps 1..4  writers, tiles round-robin: resolve the tile's prefix by
+//               look-back (a7, Eq 3), copy the ring segments to
+//               their global offsets and release ring space in tile order.
+//               Up to kMeta tiles wait for their prefix while the compute
+//               warps keep going, so the look-back latency stays hidden.
 #include "internal.cuh"
 
 namespace cuszp {
@@ -28,30 +30,50 @@ namespace cuszp {
 namespace {
 
 #ifndef CUSZP_C_STAGES
-#define CUSZP_C_STAGES 3
+#define CUSZP_C_STAGES 2
 #endif
-#ifndef CUSZP_C_STAGING
-#define CUSZP_C_STAGING 5
+#ifndef CUSZP_C_WRITERS
+#define CUSZP_C_WRITERS 2
+#endif
+#ifndef CUSZP_C_META
+#define CUSZP_C_META 8
+#endif
+#ifndef CUSZP_C_RING_WORDS
+#define CUSZP_C_RING_WORDS 1024
 #endif
 #ifndef CUSZP_C_MINBLOCKS
-#define CUSZP_C_MINBLOCKS 2
+#define CUSZP_C_MINBLOCKS 3
 #endif
-constexpr int kStages = CUSZP_C_STAGES;     // input ring depth
-constexpr int kStaging = CUSZP_C_STAGING;   // payload staging buffers = writer warps
-constexpr int kWarpWords = kBPW * kMaxBlockWords;   // 400 words per warp region
-constexpr int kFirstCompute = 1 + kStaging;         // warp index of compute warp 0
+constexpr int kStages = CUSZP_C_STAGES;          // input ring depth (16 KB tiles)
+constexpr int kWriters = CUSZP_C_WRITERS;        // scan + writer warps
+constexpr int kMeta = CUSZP_C_META;              // tiles between "computed" and "released"
+constexpr uint32_t kRing = CUSZP_C_RING_WORDS;   // words per compute-warp ring (power of 2)
+constexpr uint32_t kWarpMaxWords = kBPW * kMaxBlockWords;   // 400: worst case per warp per tile
+constexpr int kFirstCompute = 1 + kWriters;
 constexpr int kCThreads = (kFirstCompute + kComputeWarps) * 32;
+static_assert((kRing & (kRing - 1)) == 0 && kRing >= kWarpMaxWords, "ring size");
+
+struct TileMeta {
+  uint32_t tile;
+  uint32_t agg;                    // words of the tile
+  uint16_t cnt[kComputeWarps];     // words per compute warp
+  uint16_t head[kComputeWarps];    // ring position of each warp's first word
+};
 
 struct CompressSmem {
-  float in[kStages][kTileElems];                              // 48 KB
-  uint32_t words[kStaging][kComputeWarps][kWarpWords];        // 25.6 KB
-  uint32_t warp_words[kStaging][kComputeWarps];
+  float in[kStages][kTileElems];                 // 48 KB
+  uint32_t ring[kComputeWarps][kRing];           // 32 KB
+  TileMeta meta[kMeta];
   uint32_t in_tile[kStages];
-  uint32_t st_tile[kStaging];
-  uint32_t st_agg[kStaging];
-  uint32_t st_done[kStaging];      // compute warps finished with the slot's tile
-  uint64_t full[kStages], empty[kStages], staged[kStaging], freed[kStaging];
+  uint32_t meta_done[kMeta];
+  uint32_t tail[kComputeWarps];                  // ring words released (monotonic)
+  uint32_t released;                             // CTA-local tiles released (monotonic)
+  uint64_t full[kStages], empty[kStages], staged[kMeta];
 };
+
+__device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
+  return *reinterpret_cast<const volatile uint32_t*>(p);
+}
 
 // R2 op sequence with explicit RN intrinsics (never contracted); rint via the
 // 1.5*2^23 magic constant, exact for |v| < 2^22 (the R5 guard).  Returns the
@@ -62,7 +84,7 @@ struct CompressSmem {
 // the exact residual |d - r0*2eb| exceeds eb (d/2eb within an ulp of a half
 // integer), and NaN/Inf give a NaN residual: both set `rare`, and the block
 // is then redone with the full correction (quantize_exact) -- same result as
-// the oracle's sequence in every case, at 6 instructions per element.
+// the oracle's sequence in every case.
 __device__ __forceinline__ uint32_t quantize_fast(float x, float eb, float two_eb, float recip, float& vmax,
                                                   bool& rare) {
   const float v = __fmul_rn(x, recip);
@@ -135,11 +157,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kComputeWarps); }
-    for (int b = 0; b < kStaging; ++b) {
-      mbar_init(&sm.staged[b], 1);
-      mbar_init(&sm.freed[b], 1);
-      sm.st_done[b] = 0;
-    }
+    for (int m = 0; m < kMeta; ++m) { mbar_init(&sm.staged[m], 1); sm.meta_done[m] = 0; }
+    for (int w = 0; w < kComputeWarps; ++w) sm.tail[w] = 0;
+    sm.released = 0;
     fence_mbar_init();
   }
   __syncthreads();
@@ -171,15 +191,18 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         }
       }
     } else if (warp < kFirstCompute) {
-      // ------------------------------------------- writers (one per staging slot)
-      const int b = warp - 1;
-      for (uint32_t j = 0;; ++j) {
-        mbar_wait(&sm.staged[b], j & 1u);
-        const uint32_t t = sm.st_tile[b];
+      // --------------------------------------- writers (CTA-local tiles j = k, k+W, ...)
+      for (uint32_t j = uint32_t(warp - 1);; j += kWriters) {
+        const int m = int(j % kMeta);
+        const uint32_t par = (j / kMeta) & 1u;
+        while (!mbar_test(&sm.staged[m], par)) __nanosleep(128);
+        const TileMeta& md = sm.meta[m];
+        const uint32_t t = md.tile;
         if (t == kSentinel) break;
-        const uint32_t agg = sm.st_agg[b];
-        const uint32_t v = lane < kComputeWarps ? sm.warp_words[b][lane] : 0u;
-        uint32_t incl = v;
+        const uint32_t agg = md.agg;
+        const uint32_t cnt = lane < kComputeWarps ? md.cnt[lane] : 0u;
+        const uint32_t hd = lane < kComputeWarps ? md.head[lane] : 0u;
+        uint32_t incl = cnt;
 #pragma unroll
         for (int o = 1; o < kComputeWarps; o <<= 1) {
           const uint32_t y = __shfl_up_sync(kFull, incl, o);
@@ -193,41 +216,49 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           trace_put(a.trace, t, 4, global_ns());
           trace_put(a.trace, t, 5, nw);
           trace_put(a.trace, t, 6, ns);
-          uint32_t smid;
-          asm("mov.u32 %0, %smid;" : "=r"(smid));
-          trace_put(a.trace, t, 7, (uint64_t(smid) << 32) | blockIdx.x);
         }
-        // copy every compute warp's staged words to [excl + warp offset ...)
+        // a8 store: each compute warp's ring segment -> [excl + warp offset, ...)
 #pragma unroll 1
         for (int w = 0; w < kComputeWarps; ++w) {
-          const uint32_t cnt = __shfl_sync(kFull, v, w);
-          const uint32_t off = __shfl_sync(kFull, incl - v, w);
+          const uint32_t c = __shfl_sync(kFull, cnt, w);
+          const uint32_t h = __shfl_sync(kFull, hd, w);
+          const uint32_t off = __shfl_sync(kFull, incl - cnt, w);
           uint32_t* dst = payload + excl + off;
-          const uint32_t* src = sm.words[b][w];
-          for (uint32_t k = lane; k < cnt; k += 32) dst[k] = src[k];
+          const uint32_t* src = sm.ring[w];
+          for (uint32_t k = lane; k < c; k += 32) dst[k] = src[(h + k) & (kRing - 1)];
+        }
+        // release ring space in CTA tile order
+        while (ld_volatile_u32(&sm.released) != j) __nanosleep(64);
+        if (lane < kComputeWarps) sm.tail[lane] += cnt;
+        __syncwarp();
+        if (lane == 0) {
+          __threadfence_block();
+          *reinterpret_cast<volatile uint32_t*>(&sm.released) = j + 1;
         }
         __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.freed[b]);
       }
     } else {
       // ------------------------------------------------------------ compute
       const int w = warp - kFirstCompute;
       const Xpose xpose(lane);
+      uint32_t head = 0;                                // words this warp has appended (monotonic)
+      uint32_t* ring = sm.ring[w];
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
-        const int b = int(i % kStaging);
+        const int m = int(i % kMeta);
         mbar_wait(&sm.full[s], (i / kStages) & 1u);
         const uint32_t t = sm.in_tile[s];
-        if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());   // data landed
-        mbar_wait(&sm.freed[b], ((i / kStaging) & 1u) ^ 1u);   // staging slot b written out
+        if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
+        // meta slot m free (tile i - kMeta released) and room for a worst-case tile in the ring
+        while (int(i - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(32);
+        while (head + kWarpMaxWords - ld_volatile_u32(&sm.tail[w]) > kRing) __nanosleep(32);
         if (t == kSentinel) {
-          // every writer must see the sentinel: fill all slots in order
+          // every writer must see a sentinel: post one in each of the next kWriters slots
           if (w == 0 && lane == 0) {
-            for (int k = 0; k < kStaging; ++k) {
-              const int bb = int((i + k) % kStaging);
-              if (k > 0) mbar_wait(&sm.freed[bb], (((i + k) / kStaging) & 1u) ^ 1u);
-              sm.st_tile[bb] = kSentinel;
-              mbar_arrive(&sm.staged[bb]);
+            for (uint32_t k = 0; k < uint32_t(kWriters); ++k) {
+              while (int(i + k - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(64);
+              sm.meta[(i + k) % kMeta].tile = kSentinel;
+              mbar_arrive(&sm.staged[(i + k) % kMeta]);
             }
           }
           break;
@@ -235,44 +266,74 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const bool last = (t == a.num_tiles - 1);
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;   // first element of the warp
         const float* src = &sm.in[s][w * kBPW * 32];
-        uint32_t* stage = sm.words[b][w];
         uint32_t cursor = 0;
-        uint32_t fpack[4] = {0, 0, 0, 0};
+        uint32_t fpack[4];
+        // Groups of 4 blocks.  The bit transpose packs as many blocks as fit
+        // in 32 bits: 4 blocks when every v < 2^8 (F <= 7), 2 when v < 2^16,
+        // else 1.  After it, lane q*W + k holds word k of block q (W = 32 /
+        // blocks per transpose), and a ballot of the non-zero words gives every
+        // block's word count (the top plane is non-zero by definition of F).
 #pragma unroll
-        for (int p = 0; p < kBPW / 2; ++p) {
-          float xa = src[(2 * p) * 32 + lane];
-          float xb = src[(2 * p + 1) * 32 + lane];
-          if (last) {
-            if (g0 + (2 * p) * 32 + lane >= a.n) xa = 0.0f;         // virtual zero pad (R8)
-            if (g0 + (2 * p + 1) * 32 + lane >= a.n) xb = 0.0f;
+        for (int g = 0; g < kBPW / 4; ++g) {
+          float x[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            x[q] = src[(4 * g + q) * 32 + lane];
+            if (last && g0 + (4 * g + q) * 32 + lane >= a.n) x[q] = 0.0f;   // virtual zero pad (R8)
           }
-          bool rare_a, rare_b;
-          uint32_t ra = quantize_fast(xa, eb, two_eb, recip, vmax, rare_a);
-          uint32_t rb = quantize_fast(xb, eb, two_eb, recip, vmax, rare_b);
-          if (__any_sync(kFull, rare_a || rare_b)) {
-            ra = quantize_exact(xa, eb, two_eb, recip, vmax);
-            rb = quantize_exact(xb, eb, two_eb, recip, vmax);
+          uint32_t r[4];
+          bool rare = false;
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            bool rq;
+            r[q] = quantize_fast(x[q], eb, two_eb, recip, vmax, rq);
+            rare |= rq;
           }
-          const uint32_t va = lorenzo_pack(ra, lane);
-          const uint32_t vb = lorenzo_pack(rb, lane);
-          const uint32_t wa = word_count(va);
-          const uint32_t wb = word_count(vb);
-          const uint32_t oa = cursor, ob = cursor + wa;
-          cursor = ob + wb;
-          if (wa <= 16 && wb <= 16) {
-            const uint32_t tw = xpose(va | (vb << 16));
+          if (__any_sync(kFull, rare)) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
+          }
+          uint32_t v[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
+          const uint32_t span = word_count(v[0] | v[1] | v[2] | v[3]);   // max words in the group
+          uint32_t wb;      // words per block, one byte each
+          const uint32_t base = head + cursor;
+          if (span <= 8) {
+            const uint32_t tw = xpose(v[0] | (v[1] << 8) | (v[2] << 16) | (v[3] << 24));
+            const uint32_t nz = __ballot_sync(kFull, tw != 0);
+            wb = 0;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) wb |= (32u - __clz((nz >> (8 * q)) & 0xffu)) << (8 * q);
+            const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
+            const uint32_t sh = (lane >> 3) * 8, k = lane & 7;
+            if (k < ((wb >> sh) & 0xffu)) ring[(base + ((pb >> sh) & 0xffu) + k) & (kRing - 1)] = tw;
+          } else if (span <= 16) {
+            const uint32_t t01 = xpose(v[0] | (v[1] << 16));
+            const uint32_t t23 = xpose(v[2] | (v[3] << 16));
+            const uint32_t nz01 = __ballot_sync(kFull, t01 != 0), nz23 = __ballot_sync(kFull, t23 != 0);
+            const uint32_t w0 = 32u - __clz(nz01 & 0xffffu), w1 = 32u - __clz(nz01 >> 16);
+            const uint32_t w2 = 32u - __clz(nz23 & 0xffffu), w3 = 32u - __clz(nz23 >> 16);
+            wb = w0 | (w1 << 8) | (w2 << 16) | (w3 << 24);
             const bool hi = lane >= 16;
             const uint32_t k = lane & 15;
-            if (k < (hi ? wb : wa)) stage[(hi ? ob : oa) + k] = tw;
+            if (k < (hi ? w1 : w0)) ring[(base + (hi ? w0 : 0u) + k) & (kRing - 1)] = t01;
+            if (k < (hi ? w3 : w2)) ring[(base + w0 + w1 + (hi ? w2 : 0u) + k) & (kRing - 1)] = t23;
           } else {
-            const uint32_t ta = xpose(va);
-            if (uint32_t(lane) < wa) stage[oa + lane] = ta;
-            const uint32_t tb = xpose(vb);
-            if (uint32_t(lane) < wb) stage[ob + lane] = tb;
+            wb = 0;
+            uint32_t o = base;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const uint32_t tq = xpose(v[q]);
+              const uint32_t wq = 32u - __clz(__ballot_sync(kFull, tq != 0));
+              if (uint32_t(lane) < wq) ring[(o + lane) & (kRing - 1)] = tq;
+              o += wq;
+              wb |= wq << (8 * q);
+            }
           }
-          const uint32_t fa = wa ? wa - 1 : 0, fb = wb ? wb - 1 : 0;
-          const uint32_t f2 = fa | (fb << 8);
-          fpack[p >> 1] |= f2 << ((p & 1) * 16);
+          cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
+          // F = words - 1 (0 for a zero block), bytewise (counts <= 25, no carries)
+          fpack[g] = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
         }
         // F bytes of the warp's 16 blocks (Fig 12 part 1): one 16-byte store
         const uint64_t blk0 = uint64_t(t) * kTileBlocks + uint64_t(w) * kBPW;
@@ -281,27 +342,31 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         __syncwarp();
         if (lane == 0) {
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
-          sm.warp_words[b][w] = cursor;
+          TileMeta& md = sm.meta[m];
+          md.cnt[w] = uint16_t(cursor);
+          md.head[w] = uint16_t(head & (kRing - 1));
           __threadfence_block();
-          if (atomicAdd(&sm.st_done[b], 1u) == kComputeWarps - 1) {
+          if (atomicAdd(&sm.meta_done[m], 1u) == kComputeWarps - 1) {
             // last warp of the tile: aggregate -> publish at once (look-back, part 1)
             __threadfence_block();
             uint32_t agg = 0;
 #pragma unroll
-            for (int k = 0; k < kComputeWarps; ++k) agg += *reinterpret_cast<volatile uint32_t*>(&sm.warp_words[b][k]);
+            for (int k = 0; k < kComputeWarps; ++k)
+              agg += *reinterpret_cast<volatile uint16_t*>(&md.cnt[k]);
             publish_aggregate(a.status, t, agg, epoch);
             trace_put(a.trace, t, 2, global_ns());
-            sm.st_tile[b] = t;
-            sm.st_agg[b] = agg;
-            sm.st_done[b] = 0;
-            mbar_arrive(&sm.staged[b]);
+            md.tile = t;
+            md.agg = agg;
+            sm.meta_done[m] = 0;
+            mbar_arrive(&sm.staged[m]);
           }
         }
+        head += cursor;
       }
     }
   }
 
-  // R5 guard: some |d / 2eb| >= 2^22 (NaN and Inf have larger bit patterns)
+  // R5 guard: some |d / 2eb| >= 2^22 (NaN and Inf included)
   uint32_t flag = 0;
   if (!eb_ok) flag = (a.n > 0) ? kBadRange : 0u;
   else if (!(vmax < kGuard)) flag = kBadRange;

@@ -2,20 +2,22 @@
 // (paper sec 3.2 / Fig 3).
 //
 // Persistent, warp-specialised CTA:
-//   warps 0..3  producers, one per ring stage (4 tiles in flight per CTA):
-//               take a tile ticket, read the tile's 128 fixed-length bytes,
-//               turn them into block word counts (Eq 2) and tile-local
-//               offsets (warp scan), publish the tile aggregate at once,
-//               resolve the tile's global offset with the decoupled look-back
-//               (a9, Eq 3) and stream the tile's payload HBM -> shared memory
-//               with one 1D TMA bulk copy;
-//   warps 4..11 compute (stages consumed round-robin): 16 blocks each, two blocks per warp bit transpose
-//               (lane k <- word k of block A, lane 16+k <- word k of block B;
-//               afterwards lane j holds 2|l_j| + sign_j of both):
-//     a10 inverse bit-shuffle + sign,
-//     a11 inverse Lorenzo: four blocks are re-laid out through shared memory
-//         (4 consecutive elements per lane, 8 lanes per block): 3 local adds
-//         + a 3-step segmented shuffle scan,
+//   warp 0      scanner: takes a CHUNK ticket (4 tiles = 512 blocks), reads the
+//               chunk's 512 fixed-length bytes (one 16-byte load per lane),
+//               turns them into block word counts (Eq 2), per-group offsets
+//               and packing modes, publishes the chunk aggregate and resolves
+//               the chunk's global offset with the decoupled look-back (a9,
+//               Eq 3) -- one look-back per 4 tiles, overlapped with decoding
+//               through a double-buffered chunk descriptor;
+//   warp 1      loader: streams every tile's payload HBM -> shared memory
+//               with one 1D TMA bulk copy into a 4-stage ring;
+//   warps 2..9  compute, 16 blocks each in groups of 4 -- four, two or one
+//               blocks per warp bit transpose (8, 16 or 32 lanes per block):
+//     a10 inverse bit-shuffle: lane k of a block's lane range <- word k
+//         (sign map, then planes); after the transpose lane j holds
+//         v_j = 2|l_j| + sign_j of each packed block; rows go to shared memory,
+//     a11 inverse Lorenzo: 4 consecutive elements per lane, 8 lanes per block,
+//         3 local adds + a 3-step segmented shuffle scan,
 //     a12 dequantise d' = (float) r * 2eb (R13), 128-bit stores.
 // Every read is bounded by in_bytes (corrupt input -> async ECORRUPT).
 #include "internal.cuh"
@@ -31,18 +33,35 @@ namespace {
 #define CUSZP_D_STAGES 4
 #endif
 constexpr int kDStages = CUSZP_D_STAGES;
+constexpr int kChunkTiles = 4;                                  // tiles per look-back unit
+constexpr int kGroups = kTileBlocks / 4;                        // 32 decode groups per tile
 constexpr int kDataWords = kTileBlocks * kMaxBlockWords + 8;   // 3208 words: worst tile + alignment slack
-constexpr int kDThreads = (kDStages + kComputeWarps) * 32;
+constexpr int kDFirstCompute = 2;
+constexpr int kDThreads = (kDFirstCompute + kComputeWarps) * 32;
+
+struct ChunkDesc {
+  uint64_t tile_start[kChunkTiles];   // global payload word offset of each tile
+  uint32_t tile_words[kChunkTiles];
+  uint32_t gwords[kChunkTiles][kGroups];
+  uint32_t gmeta[kChunkTiles][kGroups];
+  uint32_t chunk;                     // chunk id or kSentinel
+  uint32_t ntiles;
+};
 
 struct DecompressSmem {
   uint32_t data[kDStages][kDataWords];         // 51.3 KB
-  uint16_t boff[kDStages][kTileBlocks];        // tile-local word offset of each block
-  uint8_t bwords[kDStages][kTileBlocks];       // words per block: F + 1, or 0
+  uint32_t gwords[kDStages][kGroups];          // per 4-block group: words per block, one byte each
+  uint32_t gmeta[kDStages][kGroups];           // per group: tile-local word offset | packing mode << 16
   uint32_t tile[kDStages];
   uint32_t delta[kDStages];                    // first payload word of the tile inside data[]
-  alignas(16) int scratch[kComputeWarps][8 * 32];   // per-warp 8-block re-layout for the scan
-  uint64_t full[kDStages], empty[kDStages];
+  ChunkDesc chunk[2];
+  alignas(16) uint32_t scratch[kComputeWarps][4 * 32];   // per-warp transposed rows of one group
+  uint64_t full[kDStages], empty[kDStages], chunk_ready[2], chunk_free[2];
 };
+
+__device__ __forceinline__ void lazy_wait(uint64_t* bar, uint32_t parity) {
+  while (!mbar_test(bar, parity)) __nanosleep(64);
+}
 
 }  // namespace
 
@@ -77,198 +96,245 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     }
   }
   const float two_eb = __fadd_rn(eb, eb);
+  const uint32_t num_chunks = (a.num_tiles + kChunkTiles - 1) / kChunkTiles;
   uint32_t bad = 0;
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < kDStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kComputeWarps); }
+    for (int b = 0; b < 2; ++b) { mbar_init(&sm.chunk_ready[b], 1); mbar_init(&sm.chunk_free[b], 1); }
     fence_mbar_init();
   }
   __syncthreads();
 
   if (err == CUSZP_OK && a.n > 0) {
-    if (warp < kDStages) {
-      // ------------------------------------------- producers (one per stage)
-      const int s = warp;
-      for (uint32_t j = 0;; ++j) {
-        mbar_wait(&sm.empty[s], (j & 1u) ^ 1u);
-        uint32_t t = 0;
-        if (lane == 0) t = atomicAdd(&a.ws->ticket, 1u);
-        t = __shfl_sync(kFull, t, 0);
-        if (lane == 0 && t < a.num_tiles) trace_put(a.trace, t, 0, global_ns());
-        if (t >= a.num_tiles) {
+    if (warp == 0) {
+      // ------------------------------------------------------------- scanner
+      for (uint32_t i = 0;; ++i) {
+        const int b = int(i & 1u);
+        lazy_wait(&sm.chunk_free[b], ((i >> 1) & 1u) ^ 1u);
+        ChunkDesc& cd = sm.chunk[b];
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(&a.ws->ticket, 1u);
+        c = __shfl_sync(kFull, c, 0);
+        if (c >= num_chunks) {
           if (lane == 0) {
-            sm.tile[s] = kSentinel;
-            mbar_arrive(&sm.full[s]);
+            cd.chunk = kSentinel;
+            mbar_arrive(&sm.chunk_ready[b]);
           }
           break;
         }
-        // a9: fixed lengths -> words per block (Eq 2) -> tile-local offsets
-        const uint64_t blk = uint64_t(t) * kTileBlocks + 4u * lane;   // this lane's 4 blocks
-        uint32_t fq = 0;
-        if (blk < a.nb) fq = *reinterpret_cast<const uint32_t*>(a.in + kHdr + blk);
-        uint32_t wq[4], lsum = 0;
+        const uint32_t t0 = c * kChunkTiles;
+        const uint32_t ntiles = min(uint32_t(kChunkTiles), a.num_tiles - t0);
+        // lane L: blocks 16L .. 16L+15 of the chunk = groups 4(L%8) .. +3 of tile L/8
+        const uint64_t blk = uint64_t(t0) * kTileBlocks + 16u * lane;
+        uint4 fq = make_uint4(0, 0, 0, 0);
+        if (blk < a.nb) fq = *reinterpret_cast<const uint4*>(a.in + kHdr + blk);   // in the 16-B padded F area
+        const uint32_t fw[4] = {fq.x, fq.y, fq.z, fq.w};
+        uint32_t gw[4], gspan[4], gsum[4], lsum = 0;
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          uint32_t f = (fq >> (8 * k)) & 0xffu;
-          if (blk + k >= a.nb) f = 0;
-          if (f > uint32_t(kMaxF)) { bad |= kBadCorrupt; f = 0; }
-          wq[k] = f ? f + 1 : 0;
-          lsum += wq[k];
+        for (int g = 0; g < 4; ++g) {
+          gw[g] = 0;
+          gspan[g] = 0;
+          gsum[g] = 0;
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            uint32_t f = (fw[g] >> (8 * k)) & 0xffu;
+            if (blk + 4 * g + k >= a.nb) f = 0;
+            if (f > uint32_t(kMaxF)) { bad |= kBadCorrupt; f = 0; }
+            const uint32_t wq = f ? f + 1 : 0;             // Eq 2 in 4-byte words
+            gw[g] |= wq << (8 * k);
+            gspan[g] = max(gspan[g], wq);
+            gsum[g] += wq;
+          }
+          lsum += gsum[g];
         }
+        // tile-local exclusive offsets: segmented scan over the 8 lanes of each tile
         uint32_t incl = lsum;
+        incl = uint32_t(scan_step_up(int(incl), 1, 24 << 8));
+        incl = uint32_t(scan_step_up(int(incl), 2, 24 << 8));
+        incl = uint32_t(scan_step_up(int(incl), 4, 24 << 8));
+        const int tl = lane >> 3;
+        uint32_t off = incl - lsum;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t y = __shfl_up_sync(kFull, incl, o);
-          if (lane >= o) incl += y;
+        for (int g = 0; g < 4; ++g) {
+          const uint32_t mode = gspan[g] <= 8 ? 0u : (gspan[g] <= 16 ? 1u : 2u);
+          cd.gwords[tl][4 * (lane & 7) + g] = gw[g];
+          cd.gmeta[tl][4 * (lane & 7) + g] = off | (mode << 16);
+          off += gsum[g];
         }
-        const uint32_t agg = __shfl_sync(kFull, incl, 31);
-        uint32_t o0 = incl - lsum;
-        const uint32_t o1 = o0 + wq[0], o2 = o1 + wq[1], o3 = o2 + wq[2];
-        *reinterpret_cast<uint2*>(&sm.boff[s][4 * lane]) = make_uint2(o0 | (o1 << 16), o2 | (o3 << 16));
-        *reinterpret_cast<uint32_t*>(&sm.bwords[s][4 * lane]) = wq[0] | (wq[1] << 8) | (wq[2] << 16) | (wq[3] << 24);
-        // a9: global synchronisation (decoupled look-back)
-        if (lane == 0) publish_aggregate(a.status, t, agg, epoch);
-        uint32_t nw = 0, ns = 0;
-        const uint64_t t_lb = a.trace ? global_ns() : 0;
-        const uint64_t excl = resolve_prefix(a.status, t, agg, epoch, &nw, &ns);
-        if (lane == 0 && a.trace) {
-          // decompress trace: 0 ticket, 1 F loaded + A published, 2 prefix, 3 TMA issued,
-          // 4 first compute pickup, 5 last compute done, 6 windows<<32|spins, 7 smid<<32|cta
-          trace_put(a.trace, t, 1, t_lb);
-          trace_put(a.trace, t, 2, global_ns());
-          trace_put(a.trace, t, 6, (uint64_t(nw) << 32) | ns);
-          uint32_t smid;
-          asm("mov.u32 %0, %smid;" : "=r"(smid));
-          trace_put(a.trace, t, 7, (uint64_t(smid) << 32) | blockIdx.x);
+        // tile totals and the chunk aggregate
+        uint32_t ttot[kChunkTiles], agg = 0, tpre[kChunkTiles];
+#pragma unroll
+        for (int k = 0; k < kChunkTiles; ++k) {
+          ttot[k] = __shfl_sync(kFull, incl, 8 * k + 7);
+          tpre[k] = agg;
+          agg += ttot[k];
         }
-        uint32_t tma_bytes = 0, delta = 0;
-        if (excl + agg > payload_words) {
-          bad |= kBadCorrupt;   // offsets beyond the stream: decode zeros, never read out of bounds
-          *reinterpret_cast<uint32_t*>(&sm.bwords[s][4 * lane]) = 0u;
-        } else if (agg > 0) {
-          const uint64_t start = p0 + 4 * excl, end = start + 4ull * agg;
-          const uint64_t a0 = start & ~uint64_t(15);
-          uint64_t a1 = (end + 15) & ~uint64_t(15);
-          if (a1 > a.in_bytes) a1 = a.in_bytes & ~uint64_t(15);
-          tma_bytes = uint32_t(a1 - a0);
-          delta = uint32_t(start - a0) / 4;
-          // words past the last full 16 bytes inside in_bytes (<= 3)
-          const uint64_t tail_words = end > a1 ? (end - a1) / 4 : 0;
-          if (uint64_t(lane) < tail_words)
-            sm.data[s][(a1 - a0) / 4 + lane] = *reinterpret_cast<const uint32_t*>(a.in + a1 + 4 * lane);
+        // a9: global synchronisation (decoupled look-back over chunks)
+        if (lane == 0) publish_aggregate(a.status, c, agg, epoch);
+        const uint64_t excl = resolve_prefix(a.status, c, agg, epoch);
+        const bool oob = excl + agg > payload_words;   // corrupt offsets: decode zeros, never read past in_bytes
+        if (oob) {
+          bad |= kBadCorrupt;
+#pragma unroll
+          for (int g = 0; g < 4; ++g) cd.gwords[tl][4 * (lane & 7) + g] = 0u;
+        }
+        uint64_t ts = 0;
+        uint32_t tw = 0;
+#pragma unroll
+        for (int k = 0; k < kChunkTiles; ++k)
+          if (lane == k) { ts = excl + tpre[k]; tw = oob ? 0u : ttot[k]; }
+        if (lane < kChunkTiles) {
+          cd.tile_start[lane] = ts;
+          cd.tile_words[lane] = tw;
+        }
+        if (lane == 0) {
+          cd.chunk = c;
+          cd.ntiles = ntiles;
         }
         __syncwarp();
-        if (lane == 0) {
-          sm.tile[s] = t;
-          sm.delta[s] = delta;
-          mbar_arrive_expect_tx(&sm.full[s], tma_bytes);
-          if (tma_bytes) tma_load_1d(sm.data[s], a.in + ((p0 + 4 * excl) & ~uint64_t(15)), tma_bytes, &sm.full[s]);
-          trace_put(a.trace, t, 3, global_ns());
+        if (lane == 0) mbar_arrive(&sm.chunk_ready[b]);
+      }
+    } else if (warp == 1) {
+      // -------------------------------------------------------------- loader
+      uint32_t k = 0;   // tiles issued so far (stage k % S, use k / S)
+      for (uint32_t i = 0;; ++i) {
+        const int b = int(i & 1u);
+        lazy_wait(&sm.chunk_ready[b], (i >> 1) & 1u);
+        const ChunkDesc& cd = sm.chunk[b];
+        if (cd.chunk == kSentinel) {
+          // end of work: a sentinel in every stage
+          for (int j = 0; j < kDStages; ++j, ++k) {
+            const int s = int(k % kDStages);
+            lazy_wait(&sm.empty[s], ((k / kDStages) & 1u) ^ 1u);
+            if (lane == 0) {
+              sm.tile[s] = kSentinel;
+              mbar_arrive(&sm.full[s]);
+            }
+          }
+          break;
         }
+        for (uint32_t j = 0; j < cd.ntiles; ++j, ++k) {
+          const int s = int(k % kDStages);
+          lazy_wait(&sm.empty[s], ((k / kDStages) & 1u) ^ 1u);
+          sm.gwords[s][lane] = cd.gwords[j][lane];
+          sm.gmeta[s][lane] = cd.gmeta[j][lane];
+          const uint64_t tw = cd.tile_words[j];
+          uint32_t tma_bytes = 0, delta = 0;
+          uint64_t a0 = 0;
+          if (tw > 0) {
+            const uint64_t start = p0 + 4 * cd.tile_start[j], end = start + 4 * tw;
+            a0 = start & ~uint64_t(15);
+            uint64_t a1 = (end + 15) & ~uint64_t(15);
+            if (a1 > a.in_bytes) a1 = a.in_bytes & ~uint64_t(15);
+            tma_bytes = uint32_t(a1 - a0);
+            delta = uint32_t(start - a0) / 4;
+            // words past the last full 16 bytes inside in_bytes (<= 3)
+            const uint64_t tail_words = end > a1 ? (end - a1) / 4 : 0;
+            if (uint64_t(lane) < tail_words)
+              sm.data[s][(a1 - a0) / 4 + lane] = *reinterpret_cast<const uint32_t*>(a.in + a1 + 4 * lane);
+          }
+          __syncwarp();
+          if (lane == 0) {
+            sm.tile[s] = cd.chunk * kChunkTiles + j;
+            sm.delta[s] = delta;
+            mbar_arrive_expect_tx(&sm.full[s], tma_bytes);
+            if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
+          }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.chunk_free[b]);
       }
     } else {
       // ------------------------------------------------------------ compute
-      const int w = warp - kDStages;
+      const int w = warp - kDFirstCompute;
       const Xpose xpose(lane);
-      const bool hi = lane >= 16;
-      const uint32_t k16 = lane & 15;
-      // Stages are consumed round-robin; each producer ends its stage with a
-      // sentinel, so keep going until every stage has delivered one.
-      // Each warp takes whichever stage is ready first (no head-of-line
-      // blocking behind a stage whose look-back is still waiting).
-      uint32_t phase = 0;   // bit s: parity of stage s's next phase
-      uint32_t done = 0;
-      int s = 0;
-      for (;;) {
-        // probe every pending stage once; if none is ready, sleep (in hardware)
-        // on the next pending one until it completes
-        int probes = 0;
-        while (true) {
-          if (!(done & (1u << s))) {
-            if (probes < kDStages ? mbar_test(&sm.full[s], (phase >> s) & 1u)
-                                  : mbar_try(&sm.full[s], (phase >> s) & 1u))
-              break;
-          }
-          if (++probes < kDStages || (done & (1u << s))) s = (s + 1) % kDStages;
-        }
-        phase ^= 1u << s;
+      uint32_t* scratch = sm.scratch[w];
+      for (uint32_t i = 0;; ++i) {
+        const int s = int(i % kDStages);
+        mbar_wait(&sm.full[s], (i / kDStages) & 1u);
         const uint32_t t = sm.tile[s];
-        if (t != kSentinel && lane == 0 && a.trace)
-          atomicMin(reinterpret_cast<unsigned long long*>(a.trace + 8ull * t + 4), (unsigned long long)global_ns());
-        if (t == kSentinel) {
-          done |= 1u << s;
-          if (done == (1u << kDStages) - 1) break;
-          s = (s + 1) % kDStages;
-          continue;
-        }
+        if (t == kSentinel) break;
         const bool last = (t == a.num_tiles - 1);
         const uint32_t* data = sm.data[s] + sm.delta[s];
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;
-        int* scratch = sm.scratch[w];
-        // 16 blocks = 2 rounds of 8 (4 pairs each, independent transposes in flight)
+        // 4 groups of 4 blocks: the group's words are loaded so that one bit
+        // transpose serves as many blocks as fit; the transposed rows go to
+        // scratch, from where a11/a12 continue with 4 elements per lane.
 #pragma unroll 1
-        for (int g = 0; g < kBPW / 8; ++g) {
+        for (int g = 0; g < kBPW / 4; ++g) {
+          const uint32_t wbytes = sm.gwords[s][w * 4 + g];
+          const uint32_t gm = sm.gmeta[s][w * 4 + g];
+          const uint32_t* gdata = data + (gm & 0xffffu);
+          const uint32_t mode = gm >> 16;
+          const uint32_t pbytes = wbytes * 0x01010100u;             // exclusive word prefix per block
+          int row_lane, fsh;                                         // phase-2 source for this lane
+          if (mode == 0) {
+            const uint32_t sh = (lane >> 3) * 8, kk = lane & 7;
+            const uint32_t x = kk < ((wbytes >> sh) & 0xffu) ? gdata[((pbytes >> sh) & 0xffu) + kk] : 0u;
+            scratch[lane] = xpose(x);
+            row_lane = 0;
+            fsh = 8 * (lane >> 3);
+          } else if (mode == 1) {
+            const uint32_t kk = lane & 15;
+            const uint32_t w0 = wbytes & 0xffu, w1 = (wbytes >> 8) & 0xffu;
+            const uint32_t w2 = (wbytes >> 16) & 0xffu, w3 = wbytes >> 24;
+            const bool hi = lane >= 16;
+            const uint32_t x01 = kk < (hi ? w1 : w0) ? gdata[(hi ? w0 : 0u) + kk] : 0u;
+            const uint32_t x23 = kk < (hi ? w3 : w2) ? gdata[w0 + w1 + (hi ? w2 : 0u) + kk] : 0u;
+            scratch[lane] = xpose(x01);
+            scratch[32 + lane] = xpose(x23);
+            row_lane = (lane >> 4) * 32;
+            fsh = 16 * ((lane >> 3) & 1);
+          } else {
 #pragma unroll
-          for (int h = 0; h < 4; ++h) {
-            const int lb = w * kBPW + 8 * g + 2 * h;
-            const uint32_t offs = *reinterpret_cast<const uint32_t*>(&sm.boff[s][lb]);
-            const uint32_t wds = *reinterpret_cast<const uint16_t*>(&sm.bwords[s][lb]);
-            const uint32_t oa = offs & 0xffffu, ob = offs >> 16;
-            const uint32_t wa = wds & 0xffu, wb = wds >> 8;
-            uint32_t va, vb;
-            if (wa <= 16 && wb <= 16) {
-              // a10: lane k (< 16) <- word k of A, lane 16+k <- word k of B; one transpose
-              const uint32_t idx = oa + (hi ? wa : 0u) + k16;
-              const uint32_t x = (k16 < (hi ? wb : wa)) ? data[idx] : 0u;
-              const uint32_t tw = xpose(x);
-              va = tw & 0xffffu;
-              vb = tw >> 16;
-            } else {
-              va = xpose(uint32_t(lane) < wa ? data[oa + lane] : 0u);
-              vb = xpose(uint32_t(lane) < wb ? data[ob + lane] : 0u);
+            for (int q = 0; q < 4; ++q) {
+              const uint32_t wq = (wbytes >> (8 * q)) & 0xffu, oq = (pbytes >> (8 * q)) & 0xffu;
+              scratch[32 * q + lane] = xpose(uint32_t(lane) < wq ? gdata[oq + lane] : 0u);
             }
-            // sign: v = 2|l| + s  ->  l = s ? -|l| : |l|
-            const int ma = int(va >> 1), mb = int(vb >> 1);
-            scratch[(2 * h) * 32 + lane] = (va & 1u) ? -ma : ma;
-            scratch[(2 * h + 1) * 32 + lane] = (vb & 1u) ? -mb : mb;
+            row_lane = (lane >> 3) * 32;
+            fsh = 0;
           }
           __syncwarp();
-          // a11: 8 blocks, 4 consecutive elements per lane, 8 lanes per block, 2 passes
-#pragma unroll
-          for (int q = 0; q < 2; ++q) {
-            int4 e = *reinterpret_cast<const int4*>(&scratch[(4 * q + (lane >> 3)) * 32 + 4 * (lane & 7)]);
-            e.y += e.x;
-            e.z += e.y;
-            e.w += e.z;
-            int incl = e.w;
-            incl = scan_step_up(incl, 1, 24 << 8);
-            incl = scan_step_up(incl, 2, 24 << 8);
-            incl = scan_step_up(incl, 4, 24 << 8);
-            const int carry = incl - e.w;
-            e.x += carry; e.y += carry; e.z += carry; e.w += carry;
-            // a12: d' = r * 2eb
-            float4 d;
-            d.x = __fmul_rn(__int2float_rn(e.x), two_eb);
-            d.y = __fmul_rn(__int2float_rn(e.y), two_eb);
-            d.z = __fmul_rn(__int2float_rn(e.z), two_eb);
-            d.w = __fmul_rn(__int2float_rn(e.w), two_eb);
-            const uint64_t i0 = g0 + uint64_t(8 * g + 4 * q + (lane >> 3)) * 32 + 4 * (lane & 7);
-            if (!last || i0 + 4 <= a.n) {
-              *reinterpret_cast<float4*>(a.out + i0) = d;
-            } else {
-              if (i0 < a.n) a.out[i0] = d.x;
-              if (i0 + 1 < a.n) a.out[i0 + 1] = d.y;
-              if (i0 + 2 < a.n) a.out[i0 + 2] = d.z;
-            }
+          const uint32_t fmask = mode == 0 ? 0xffu : (mode == 1 ? 0xffffu : 0xffffffffu);
+          const uint4 raw = *reinterpret_cast<const uint4*>(&scratch[row_lane + 4 * (lane & 7)]);
+          int4 e;
+          {
+            const uint32_t v0 = (raw.x >> fsh) & fmask, v1 = (raw.y >> fsh) & fmask;
+            const uint32_t v2 = (raw.z >> fsh) & fmask, v3 = (raw.w >> fsh) & fmask;
+            e.x = (v0 & 1u) ? -int(v0 >> 1) : int(v0 >> 1);   // l = sign ? -|l| : |l|
+            e.y = (v1 & 1u) ? -int(v1 >> 1) : int(v1 >> 1);
+            e.z = (v2 & 1u) ? -int(v2 >> 1) : int(v2 >> 1);
+            e.w = (v3 & 1u) ? -int(v3 >> 1) : int(v3 >> 1);
+          }
+          // a11: r_j = sum_{i <= j} l_i within the block
+          e.y += e.x;
+          e.z += e.y;
+          e.w += e.z;
+          int incl = e.w;
+          incl = scan_step_up(incl, 1, 24 << 8);
+          incl = scan_step_up(incl, 2, 24 << 8);
+          incl = scan_step_up(incl, 4, 24 << 8);
+          const int carry = incl - e.w;
+          e.x += carry; e.y += carry; e.z += carry; e.w += carry;
+          // a12: d' = r * 2eb
+          float4 d;
+          d.x = __fmul_rn(__int2float_rn(e.x), two_eb);
+          d.y = __fmul_rn(__int2float_rn(e.y), two_eb);
+          d.z = __fmul_rn(__int2float_rn(e.z), two_eb);
+          d.w = __fmul_rn(__int2float_rn(e.w), two_eb);
+          const uint64_t i0 = g0 + uint64_t(4 * g + (lane >> 3)) * 32 + 4 * (lane & 7);
+          if (!last || i0 + 4 <= a.n) {
+            *reinterpret_cast<float4*>(a.out + i0) = d;
+          } else {
+            if (i0 < a.n) a.out[i0] = d.x;
+            if (i0 + 1 < a.n) a.out[i0 + 1] = d.y;
+            if (i0 + 2 < a.n) a.out[i0 + 2] = d.z;
           }
           __syncwarp();
         }
         __syncwarp();
-        if (lane == 0) {
-          if (a.trace) atomicMax(reinterpret_cast<unsigned long long*>(a.trace + 8ull * t + 5), (unsigned long long)global_ns());
-          mbar_arrive(&sm.empty[s]);
-        }
-        s = (s + 1) % kDStages;
+        if (lane == 0) mbar_arrive(&sm.empty[s]);
       }
     }
   }
@@ -278,8 +344,8 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     if (threadIdx.x == 0 && final_status == CUSZP_OK) {
       const uint32_t acc = *reinterpret_cast<volatile uint32_t*>(&a.ws->status_accum);
       if (acc & kBadCorrupt) final_status = CUSZP_ECORRUPT;
-      if (final_status == CUSZP_OK && a.num_tiles > 0 && a.n > 0) {
-        const uint64_t total = ld_relaxed_u64(a.status + a.num_tiles - 1) & kValueMask;
+      if (final_status == CUSZP_OK && num_chunks > 0 && a.n > 0) {
+        const uint64_t total = ld_relaxed_u64(a.status + num_chunks - 1) & kValueMask;
         if (total != payload_words) final_status = CUSZP_ECORRUPT;
       }
     }

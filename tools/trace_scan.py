@@ -95,7 +95,7 @@ def main():
     ob = torch.zeros(1, dtype=torch.int64, device=dev)
     mm = torch.empty(2, dtype=torch.float32, device=dev)
     y = torch.empty(n, dtype=torch.float32, device=dev)
-    trace = torch.zeros(nt * 8, dtype=torch.int64, device=dev)
+    trace = torch.zeros(nt * 16, dtype=torch.int64, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     sp = torch.cuda.current_stream().cuda_stream
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
@@ -110,15 +110,20 @@ def main():
         ev[1].record()
         if traced:
             torch.cuda.synchronize()
-            trc = trace.view(nt, 8).cpu().numpy().astype(np.int64)
+            trc = trace[: nt * 8].view(nt, 8).cpu().numpy().astype(np.int64)
             trace.zero_()
-            trace.view(nt, 8)[:, 4] = (1 << 62)
+            trace[: nt * 8].view(nt, 8)[:, 4] = (1 << 62)
         flush.zero_()
         ev[2].record()
         h.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.data_ptr(), ws.numel(), sp)
         torch.cuda.synchronize()
     h.cuszp_debug_set_trace(None)
-    trd = trace.view(nt, 8).cpu().numpy().astype(np.int64)
+    trd = trace[: nt * 8].view(nt, 8).cpu().numpy().astype(np.int64)
+    pw = trace[nt * 8:].view(nt, 8).cpu().numpy().astype(np.int64)
+    last = np.argmax(pw, axis=1)
+    spread = (pw.max(axis=1) - pw.min(axis=1)) / 1e3
+    print("decompress: which compute warp finishes a tile last:", np.bincount(last, minlength=8).tolist(),
+          " spread first..last warp (us):", pct(spread))
     S = int(ob.item())
     print(f"n={n} tiles={nt} S={S} CR={4 * n / S:.2f}  compress {ev[0].elapsed_time(ev[1]) * 1e3:.1f} us")
     report("compress", trc, ev[0].elapsed_time(ev[1]) * 1e6)
