@@ -140,18 +140,20 @@ void oracle_value_range(const float* x, size_t n, float* mn, float* mx) {
 int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q) {
   /* r_i = round(d_i / 2eb), guaranteeing |r_i * 2eb - d_i| <= eb.
    * fp32 op sequence R2 (shared by definition, not by code, with the GPU):
-   *   two_eb = eb + eb; recip = 1 / two_eb           (once)
-   *   v  = d * recip                                   (RN)
-   *   r0 = rint(v)                                     (half-to-even)
+   *   two_eb = eb + eb; recip = 1 / two_eb           (fp32, once)
+   *   r0  = nearest integer (ties to even) to the EXACT product d * recip
+   *         -- one rounding; the product of two floats is exact in double
+   *   guard: |r0| < 2^22, else ERANGE (R5; NaN and Inf fail it)
    *   res = fmaf(-r0, two_eb, d)   -- exact, see DESIGN R2
-   *   r  = r0 + (res > eb) - (res < -eb)   -> |d - r*2eb| <= eb exactly  */
+   *   r   = r0 + (res > eb) - (res < -eb)   -> |d - r*2eb| <= eb exactly  */
   std::fesetround(FE_TONEAREST);
   const float two_eb = eb_abs + eb_abs;
   const float recip = 1.0f / two_eb;
   for (size_t i = 0; i < n; ++i) {
-    const float v = x[i] * recip;
-    if (!(std::fabs(v) < GUARD)) return ORACLE_ERANGE;  /* NaN/Inf/overflow, R5 */
-    const float r0 = std::nearbyint(v);
+    const double p = double(x[i]) * double(recip);      /* exact */
+    const double r0d = std::nearbyint(p);
+    if (!(std::fabs(r0d) < double(GUARD))) return ORACLE_ERANGE;
+    const float r0 = float(r0d);                         /* exact, |r0| < 2^22 */
     const float res = std::fmaf(-r0, two_eb, x[i]);
     int32_t r = int32_t(r0);
     if (res > eb_abs) r += 1;

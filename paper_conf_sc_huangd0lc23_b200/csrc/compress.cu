@@ -33,13 +33,16 @@ namespace {
 #define CUSZP_C_STAGES 2
 #endif
 #ifndef CUSZP_C_WRITERS
-#define CUSZP_C_WRITERS 2
+#define CUSZP_C_WRITERS 3
 #endif
 #ifndef CUSZP_C_META
 #define CUSZP_C_META 8
 #endif
 #ifndef CUSZP_C_RING_WORDS
 #define CUSZP_C_RING_WORDS 1024
+#endif
+#ifndef CUSZP_C_POLL_NS
+#define CUSZP_C_POLL_NS 32
 #endif
 #ifndef CUSZP_C_MINBLOCKS
 #define CUSZP_C_MINBLOCKS 3
@@ -48,10 +51,9 @@ constexpr int kStages = CUSZP_C_STAGES;          // input ring depth (16 KB tile
 constexpr int kWriters = CUSZP_C_WRITERS;        // scan + writer warps
 constexpr int kMeta = CUSZP_C_META;              // tiles between "computed" and "released"
 constexpr uint32_t kRing = CUSZP_C_RING_WORDS;   // words per compute-warp ring (power of 2)
-constexpr uint32_t kWarpMaxWords = kBPW * kMaxBlockWords;   // 400: worst case per warp per tile
 constexpr int kFirstCompute = 1 + kWriters;
 constexpr int kCThreads = (kFirstCompute + kComputeWarps) * 32;
-static_assert((kRing & (kRing - 1)) == 0 && kRing >= kWarpMaxWords, "ring size");
+static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * kMaxBlockWords, "ring size");
 
 struct TileMeta {
   uint32_t tile;
@@ -75,32 +77,31 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
   return *reinterpret_cast<const volatile uint32_t*>(p);
 }
 
-// R2 op sequence with explicit RN intrinsics (never contracted); rint via the
-// 1.5*2^23 magic constant, exact for |v| < 2^22 (the R5 guard).  Returns the
-// quantisation integer r BIASED by the magic's bit pattern (r + 0x4B400000),
-// which the Lorenzo step removes for free.
+// R2 op sequence with explicit RN intrinsics (never contracted further):
+// t = fma(d, recip, 1.5*2^23) rounds the exact product d*recip to the nearest
+// integer (ties to even) in ONE rounding for |d*recip| < 2^22; r0 = t - 1.5*2^23
+// is exact.  Returns the quantisation integer r BIASED by the magic's bit
+// pattern (r + 0x4B400000), which the Lorenzo step removes for free.
 //
-// Fast path: r0 = rint(d * recip).  It differs from round(d / 2eb) only when
-// the exact residual |d - r0*2eb| exceeds eb (d/2eb within an ulp of a half
-// integer), and NaN/Inf give a NaN residual: both set `rare`, and the block
-// is then redone with the full correction (quantize_exact) -- same result as
-// the oracle's sequence in every case.
-__device__ __forceinline__ uint32_t quantize_fast(float x, float eb, float two_eb, float recip, float& vmax,
+// Fast path: r0.  It differs from round(d / 2eb) only when the exact residual
+// |d - r0*2eb| exceeds eb (d/2eb within an ulp of a half integer), and
+// NaN/Inf give a NaN residual: both set `rare`, and the group is then redone
+// with the full correction (quantize_exact) -- the oracle's sequence in every
+// case.  The R5 guard |r0| < 2^22 is tracked as a running max of |r0|.
+__device__ __forceinline__ uint32_t quantize_fast(float x, float eb, float two_eb, float recip, float& rmax,
                                                   bool& rare) {
-  const float v = __fmul_rn(x, recip);
-  vmax = fmaxf(vmax, fabsf(v));                    // R5 guard (|v| >= 2^22, Inf); NaN -> `rare`
-  const float t = __fadd_rn(v, kRoundMagic);
+  const float t = __fmaf_rn(x, recip, kRoundMagic);
   const float r0 = __fsub_rn(t, kRoundMagic);
+  rmax = fmaxf(rmax, fabsf(r0));                   // R5 guard (|r0| >= 2^22, Inf); NaN -> `rare`
   const float res = __fmaf_rn(-r0, two_eb, x);     // exact residual (R2)
   rare = !(fabsf(res) <= eb);
   return __float_as_uint(t);
 }
 
-__device__ __forceinline__ uint32_t quantize_exact(float x, float eb, float two_eb, float recip, float& vmax) {
-  const float v = __fmul_rn(x, recip);
-  if (!(fabsf(v) < kGuard)) vmax = __int_as_float(0x7f800000);   // NaN too
-  const float t = __fadd_rn(v, kRoundMagic);
+__device__ __forceinline__ uint32_t quantize_exact(float x, float eb, float two_eb, float recip, float& rmax) {
+  const float t = __fmaf_rn(x, recip, kRoundMagic);
   const float r0 = __fsub_rn(t, kRoundMagic);
+  if (!(fabsf(r0) < kGuard)) rmax = __int_as_float(0x7f800000);   // NaN too
   const float res = __fmaf_rn(-r0, two_eb, x);
   uint32_t r = __float_as_uint(t);
   r += uint32_t(int(res > eb) - int(res < -eb));
@@ -151,7 +152,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   const float two_eb = __fadd_rn(eb, eb);
   const bool eb_ok = (eb >= kFltMin) && isfinite(two_eb) && a.n > 0;   // R5
   const float recip = __fdiv_rn(1.0f, two_eb);
-  float vmax = 0.0f;        // max over this thread's elements of |d / 2eb| (R5 guard)
+  float vmax = 0.0f;        // max over this thread's elements of |r0| (R5 guard)
   const uint64_t p0 = kHdr + align16(a.nb);
   uint32_t* payload = reinterpret_cast<uint32_t*>(a.out + p0);
 
@@ -195,7 +196,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t j = uint32_t(warp - 1);; j += kWriters) {
         const int m = int(j % kMeta);
         const uint32_t par = (j / kMeta) & 1u;
-        while (!mbar_test(&sm.staged[m], par)) __nanosleep(128);
+        while (!mbar_test(&sm.staged[m], par)) __nanosleep(4 * CUSZP_C_POLL_NS);
         const TileMeta& md = sm.meta[m];
         const uint32_t t = md.tile;
         if (t == kSentinel) break;
@@ -246,12 +247,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
-        mbar_wait(&sm.full[s], (i / kStages) & 1u);
+        while (!mbar_test(&sm.full[s], (i / kStages) & 1u)) __nanosleep(CUSZP_C_POLL_NS);
         const uint32_t t = sm.in_tile[s];
         if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
-        // meta slot m free (tile i - kMeta released) and room for a worst-case tile in the ring
-        while (int(i - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(32);
-        while (head + kWarpMaxWords - ld_volatile_u32(&sm.tail[w]) > kRing) __nanosleep(32);
+        // meta slot m free (tile i - kMeta released)
+        while (int(i - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(CUSZP_C_POLL_NS);
         if (t == kSentinel) {
           // every writer must see a sentinel: post one in each of the next kWriters slots
           if (w == 0 && lane == 0) {
@@ -296,6 +296,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           uint32_t v[4];
 #pragma unroll
           for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
+          // room in this warp's ring for a worst-case group (4 x 25 words)
+          while (head + cursor + 4 * kMaxBlockWords - ld_volatile_u32(&sm.tail[w]) > kRing)
+            __nanosleep(CUSZP_C_POLL_NS);
           const uint32_t span = word_count(v[0] | v[1] | v[2] | v[3]);   // max words in the group
           uint32_t wb;      // words per block, one byte each
           const uint32_t base = head + cursor;
@@ -366,7 +369,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
     }
   }
 
-  // R5 guard: some |d / 2eb| >= 2^22 (NaN and Inf included)
+  // R5 guard: some |r0| >= 2^22 (NaN and Inf included)
   uint32_t flag = 0;
   if (!eb_ok) flag = (a.n > 0) ? kBadRange : 0u;
   else if (!(vmax < kGuard)) flag = kBadRange;

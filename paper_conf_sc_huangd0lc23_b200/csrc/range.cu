@@ -8,6 +8,10 @@
 // the accumulators to their identity 0 (so the workspace needs no memset).
 #include "internal.cuh"
 
+#ifndef CUSZP_RANGE_UNROLL
+#define CUSZP_RANGE_UNROLL 4
+#endif
+
 namespace cuszp {
 
 namespace {
@@ -33,7 +37,7 @@ __global__ void __launch_bounds__(256) range_kernel(RangeArgs a) {
   if (aligned) {
     const uint64_t n4 = a.n / 4;
     const float4* in4 = reinterpret_cast<const float4*>(a.in);
-    constexpr int U = 4;
+    constexpr int U = CUSZP_RANGE_UNROLL;
     uint64_t i = tid;
     for (; i + (U - 1) * nthreads < n4; i += U * nthreads) {
       float4 v[U];

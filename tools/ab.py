@@ -46,8 +46,8 @@ def main():
     y = torch.empty(n, dtype=torch.float32, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     sp = torch.cuda.current_stream().cuda_stream
-    ev = [torch.cuda.Event(enable_timing=True) for _ in range(6)]
-    res = {i: {"range": [], "compress": [], "decompress": []} for i in range(len(libs))}
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(9)]
+    res = {i: {"range": [], "compress": [], "decompress": [], "rel_chain": []} for i in range(len(libs))}
     ref = None
     for r in range(a.rounds + 2):
         for i, h in enumerate(libs):
@@ -59,6 +59,11 @@ def main():
                                     ws.data_ptr(), ws.numel(), sp); ev[3].record()
             flush.zero_(); ev[4].record()
             h.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.data_ptr(), ws.numel(), sp); ev[5].record()
+            # REL chain as the product runs it: flush, range, compress (no flush between)
+            flush.zero_(); ev[6].record()
+            h.cuszp_range(x.data_ptr(), n, mm.data_ptr(), ws.data_ptr(), ws.numel(), sp)
+            h.cuszp_compress_minmax(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, out.data_ptr(), cap, ob.data_ptr(),
+                                    ws.data_ptr(), ws.numel(), sp); ev[7].record()
             torch.cuda.synchronize()
             S = int(ob.item())
             digest = (S, float(y[:1000].sum()), float(y[-1000:].sum()))
@@ -68,12 +73,14 @@ def main():
                 res[i]["range"].append(ev[0].elapsed_time(ev[1]) * 1e3)
                 res[i]["compress"].append(ev[2].elapsed_time(ev[3]) * 1e3)
                 res[i]["decompress"].append(ev[4].elapsed_time(ev[5]) * 1e3)
+                res[i]["rel_chain"].append(ev[6].elapsed_time(ev[7]) * 1e3)
     print(f"n={n} S={ref[0]} CR={4 * n / ref[0]:.2f}  (us: median / min)")
     for i, p in enumerate(a.libs):
         d = res[i]
         print(f"{os.path.basename(p):40s} range {np.median(d['range']):7.1f}/{min(d['range']):7.1f}  "
               f"compress {np.median(d['compress']):7.1f}/{min(d['compress']):7.1f}  "
-              f"decompress {np.median(d['decompress']):7.1f}/{min(d['decompress']):7.1f}")
+              f"decompress {np.median(d['decompress']):7.1f}/{min(d['decompress']):7.1f}  "
+              f"range+compress {np.median(d['rel_chain']):7.1f}")
 
 
 if __name__ == "__main__":
