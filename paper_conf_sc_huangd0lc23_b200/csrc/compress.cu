@@ -98,6 +98,27 @@ __device__ __forceinline__ uint32_t quantize_fast(float x, float eb, float two_e
   return __float_as_uint(t);
 }
 
+// Two elements at once with the packed fp32 pipe (FFMA2 / FADD2; same IEEE
+// RN semantics per element as the scalar sequence above).  Returns the two
+// biased integers; updates the running max |r0| (guard) and max |res|.
+__device__ __forceinline__ void quantize_fast2(float xa, float xb, float two_eb, float recip, float& rmax,
+                                               float& resmax, uint32_t& ta, uint32_t& tb) {
+  uint64_t x, t, r0, res;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(x) : "f"(xa), "f"(xb));
+  const uint64_t rc = (uint64_t(__float_as_uint(recip)) << 32) | __float_as_uint(recip);
+  const uint64_t mg = (uint64_t(__float_as_uint(kRoundMagic)) << 32) | __float_as_uint(kRoundMagic);
+  const uint64_t nt = (uint64_t(__float_as_uint(-two_eb)) << 32) | __float_as_uint(-two_eb);
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(t) : "l"(x), "l"(rc), "l"(mg));
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r0) : "l"(t), "l"(mg));
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(res) : "l"(r0), "l"(nt), "l"(x));
+  float r0a, r0b, ra, rb;
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(r0a), "=f"(r0b) : "l"(r0));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(ra), "=f"(rb) : "l"(res));
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(ta), "=r"(tb) : "l"(t));
+  rmax = fmaxf(rmax, fmaxf(fabsf(r0a), fabsf(r0b)));       // R5 guard on finite values (Inf too)
+  resmax = fmaxf(resmax, fmaxf(fabsf(ra), fabsf(rb)));
+}
+
 __device__ __forceinline__ uint32_t quantize_exact(float x, float eb, float two_eb, float recip, float& rmax) {
   const float t = __fmaf_rn(x, recip, kRoundMagic);
   const float r0 = __fsub_rn(t, kRoundMagic);
@@ -153,6 +174,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   const bool eb_ok = (eb >= kFltMin) && isfinite(two_eb) && a.n > 0;   // R5
   const float recip = __fdiv_rn(1.0f, two_eb);
   float vmax = 0.0f;        // max over this thread's elements of |r0| (R5 guard)
+  uint32_t wmax = 0;        // max words of any block (> 25 only for NaN/Inf data)
   const uint64_t p0 = kHdr + align16(a.nb);
   uint32_t* payload = reinterpret_cast<uint32_t*>(a.out + p0);
 
@@ -282,14 +304,12 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             if (last && g0 + (4 * g + q) * 32 + lane >= a.n) x[q] = 0.0f;   // virtual zero pad (R8)
           }
           uint32_t r[4];
-          bool rare = false;
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            bool rq;
-            r[q] = quantize_fast(x[q], eb, two_eb, recip, vmax, rq);
-            rare |= rq;
-          }
-          if (__any_sync(kFull, rare)) {
+          float resmax = 0.0f;
+          quantize_fast2(x[0], x[1], two_eb, recip, vmax, resmax, r[0], r[1]);
+          quantize_fast2(x[2], x[3], two_eb, recip, vmax, resmax, r[2], r[3]);
+          // NaN residuals are not caught here (fmax drops NaN) but NaN/Inf data
+          // always yield a block with > 25 words below (flagged, R5)
+          if (__any_sync(kFull, resmax > eb)) {
 #pragma unroll
             for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
           }
@@ -299,43 +319,44 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           // room in this warp's ring for a worst-case group (4 x 25 words)
           while (head + cursor + 4 * kMaxBlockWords - ld_volatile_u32(&sm.tail[w]) > kRing)
             __nanosleep(CUSZP_C_POLL_NS);
-          const uint32_t span = word_count(v[0] | v[1] | v[2] | v[3]);   // max words in the group
-          uint32_t wb;      // words per block, one byte each
+#ifdef CUSZP_DIAG_TINY
+          v[0] = v[1] = v[2] = v[3] = 0;   // diagnostics only: all zero blocks (wrong output)
+#endif
+          // a5: words per block = bit length of the block's OR of v (= of its max)
+          uint32_t wq[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            uint32_t b;
+            asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(__reduce_or_sync(kFull, v[q])));   // -1 for 0
+            wq[q] = b + 1;
+          }
+          const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+          wmax = max(wmax, span);                                        // > 25: NaN/Inf data (R5)
+          const uint32_t wb = wq[0] | (wq[1] << 8) | (wq[2] << 16) | (wq[3] << 24);
           const uint32_t base = head + cursor;
           if (span <= 8) {
             const uint32_t tw = xpose(v[0] | (v[1] << 8) | (v[2] << 16) | (v[3] << 24));
-            const uint32_t nz = __ballot_sync(kFull, tw != 0);
-            wb = 0;
-#pragma unroll
-            for (int q = 0; q < 4; ++q) wb |= (32u - __clz((nz >> (8 * q)) & 0xffu)) << (8 * q);
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
-            const uint32_t sh = (lane >> 3) * 8, k = lane & 7;
-            if (k < ((wb >> sh) & 0xffu)) ring[(base + ((pb >> sh) & 0xffu) + k) & (kRing - 1)] = tw;
+            const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
+            if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;
           } else if (span <= 16) {
             const uint32_t t01 = xpose(v[0] | (v[1] << 16));
             const uint32_t t23 = xpose(v[2] | (v[3] << 16));
-            const uint32_t nz01 = __ballot_sync(kFull, t01 != 0), nz23 = __ballot_sync(kFull, t23 != 0);
-            const uint32_t w0 = 32u - __clz(nz01 & 0xffffu), w1 = 32u - __clz(nz01 >> 16);
-            const uint32_t w2 = 32u - __clz(nz23 & 0xffffu), w3 = 32u - __clz(nz23 >> 16);
-            wb = w0 | (w1 << 8) | (w2 << 16) | (w3 << 24);
             const bool hi = lane >= 16;
             const uint32_t k = lane & 15;
-            if (k < (hi ? w1 : w0)) ring[(base + (hi ? w0 : 0u) + k) & (kRing - 1)] = t01;
-            if (k < (hi ? w3 : w2)) ring[(base + w0 + w1 + (hi ? w2 : 0u) + k) & (kRing - 1)] = t23;
+            if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;
+            if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;
           } else {
-            wb = 0;
             uint32_t o = base;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
               const uint32_t tq = xpose(v[q]);
-              const uint32_t wq = 32u - __clz(__ballot_sync(kFull, tq != 0));
-              if (uint32_t(lane) < wq) ring[(o + lane) & (kRing - 1)] = tq;
-              o += wq;
-              wb |= wq << (8 * q);
+              if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;
+              o += wq[q];
             }
           }
           cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
-          // F = words - 1 (0 for a zero block), bytewise (counts <= 25, no carries)
+          // F = words - 1 (0 for a zero block), bytewise (counts <= 32, no carries)
           fpack[g] = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
         }
         // F bytes of the warp's 16 blocks (Fig 12 part 1): one 16-byte store
@@ -372,7 +393,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   // R5 guard: some |r0| >= 2^22 (NaN and Inf included)
   uint32_t flag = 0;
   if (!eb_ok) flag = (a.n > 0) ? kBadRange : 0u;
-  else if (!(vmax < kGuard)) flag = kBadRange;
+  else if (!(vmax < kGuard) || wmax > uint32_t(kMaxBlockWords)) flag = kBadRange;
 
   if (cta_finish(a.ws, flag)) {
     uint32_t final_status = CUSZP_OK;

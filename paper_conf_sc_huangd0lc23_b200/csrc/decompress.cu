@@ -50,18 +50,19 @@ struct ChunkDesc {
 
 struct DecompressSmem {
   uint32_t data[kDStages][kDataWords];         // 51.3 KB
-  uint32_t gwords[kDStages][kGroups];          // per 4-block group: words per block, one byte each
-  uint32_t gmeta[kDStages][kGroups];           // per group: tile-local word offset | packing mode << 16
+  uint2 ginfo[kDStages][kGroups];              // per 4-block group: {words per block (bytes), offset | mode << 16}
   uint32_t tile[kDStages];
   uint32_t delta[kDStages];                    // first payload word of the tile inside data[]
   ChunkDesc chunk[2];
   alignas(16) uint32_t scratch[kComputeWarps][4 * 32];   // per-warp transposed rows of one group
-  uint64_t full[kDStages], empty[kDStages], chunk_ready[2], chunk_free[2];
+  uint64_t full[kDStages];                     // TMA completion (the only mbarriers)
 };
 
-__device__ __forceinline__ void lazy_wait(uint64_t* bar, uint32_t parity) {
-  while (!mbar_test(bar, parity)) __nanosleep(64);
-}
+// named barriers (id 0 is __syncthreads)
+constexpr uint32_t kBarFull0 = 1, kBarEmpty0 = kBarFull0 + kDStages;
+constexpr uint32_t kBarReady0 = kBarEmpty0 + kDStages, kBarFree0 = kBarReady0 + 2;
+constexpr uint32_t kBarCount = 32 + 32 * kComputeWarps;   // loader + compute warps
+static_assert(kBarFree0 + 2 <= 16, "named barriers");
 
 }  // namespace
 
@@ -100,8 +101,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
   uint32_t bad = 0;
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kDStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kComputeWarps); }
-    for (int b = 0; b < 2; ++b) { mbar_init(&sm.chunk_ready[b], 1); mbar_init(&sm.chunk_free[b], 1); }
+    for (int s = 0; s < kDStages; ++s) mbar_init(&sm.full[s], 1);
     fence_mbar_init();
   }
   __syncthreads();
@@ -111,16 +111,14 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
       // ------------------------------------------------------------- scanner
       for (uint32_t i = 0;; ++i) {
         const int b = int(i & 1u);
-        lazy_wait(&sm.chunk_free[b], ((i >> 1) & 1u) ^ 1u);
+        if (i >= 2) named_sync(kBarFree0 + b, 64);
         ChunkDesc& cd = sm.chunk[b];
         uint32_t c = 0;
         if (lane == 0) c = atomicAdd(&a.ws->ticket, 1u);
         c = __shfl_sync(kFull, c, 0);
         if (c >= num_chunks) {
-          if (lane == 0) {
-            cd.chunk = kSentinel;
-            mbar_arrive(&sm.chunk_ready[b]);
-          }
+          if (lane == 0) cd.chunk = kSentinel;
+          named_arrive(kBarReady0 + b, 64);
           break;
         }
         const uint32_t t0 = c * kChunkTiles;
@@ -192,33 +190,39 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           cd.chunk = c;
           cd.ntiles = ntiles;
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.chunk_ready[b]);
+        named_arrive(kBarReady0 + b, 64);
       }
     } else if (warp == 1) {
       // -------------------------------------------------------------- loader
-      uint32_t k = 0;   // tiles issued so far (stage k % S, use k / S)
+      // Tile k goes to stage k % S once the compute warps released it (named
+      // barrier EMPTY); one step behind, the loader waits for tile k-1's TMA
+      // bytes and signals the compute warps (named barrier FULL).
+      uint32_t k = 0;              // tiles loaded so far
+      bool prev_pending = false;   // tile k-1 loaded, not yet signalled
+      auto signal_prev = [&]() {
+        if (prev_pending) {
+          const int sp = int((k - 1) % kDStages);
+          mbar_wait(&sm.full[sp], ((k - 1) / kDStages) & 1u);
+          named_arrive(kBarFull0 + sp, kBarCount);
+          prev_pending = false;
+        }
+      };
       for (uint32_t i = 0;; ++i) {
         const int b = int(i & 1u);
-        lazy_wait(&sm.chunk_ready[b], (i >> 1) & 1u);
+        named_sync(kBarReady0 + b, 64);
         const ChunkDesc& cd = sm.chunk[b];
         if (cd.chunk == kSentinel) {
-          // end of work: a sentinel in every stage
-          for (int j = 0; j < kDStages; ++j, ++k) {
-            const int s = int(k % kDStages);
-            lazy_wait(&sm.empty[s], ((k / kDStages) & 1u) ^ 1u);
-            if (lane == 0) {
-              sm.tile[s] = kSentinel;
-              mbar_arrive(&sm.full[s]);
-            }
-          }
+          signal_prev();
+          const int s = int(k % kDStages);
+          if (k >= uint32_t(kDStages)) named_sync(kBarEmpty0 + s, kBarCount);
+          if (lane == 0) sm.tile[s] = kSentinel;
+          named_arrive(kBarFull0 + s, kBarCount);
           break;
         }
-        for (uint32_t j = 0; j < cd.ntiles; ++j, ++k) {
+        for (uint32_t j = 0; j < cd.ntiles; ++j) {
           const int s = int(k % kDStages);
-          lazy_wait(&sm.empty[s], ((k / kDStages) & 1u) ^ 1u);
-          sm.gwords[s][lane] = cd.gwords[j][lane];
-          sm.gmeta[s][lane] = cd.gmeta[j][lane];
+          if (k >= uint32_t(kDStages)) named_sync(kBarEmpty0 + s, kBarCount);
+          sm.ginfo[s][lane] = make_uint2(cd.gwords[j][lane], cd.gmeta[j][lane]);
           const uint64_t tw = cd.tile_words[j];
           uint32_t tma_bytes = 0, delta = 0;
           uint64_t a0 = 0;
@@ -238,103 +242,110 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           if (lane == 0) {
             sm.tile[s] = cd.chunk * kChunkTiles + j;
             sm.delta[s] = delta;
-            mbar_arrive_expect_tx(&sm.full[s], tma_bytes);
+            mbar_arrive_expect_tx(&sm.full[s], tma_bytes);   // one phase per use, even with 0 bytes
             if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
           }
+          signal_prev();
+          prev_pending = true;
+          ++k;
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.chunk_free[b]);
+        named_arrive(kBarFree0 + b, 64);
       }
     } else {
       // ------------------------------------------------------------ compute
       const int w = warp - kDFirstCompute;
       const Xpose xpose(lane);
       uint32_t* scratch = sm.scratch[w];
+      // per-lane constants: quad mode -> block q = lane/8 owns lanes 8q..8q+7;
+      // pair mode -> blocks (0,1) in lanes 0-15 / 16-31 of row 0, (2,3) of row 1
+      const uint32_t q = uint32_t(lane) >> 3, k8 = lane & 7, k16 = lane & 15;
+      const bool hi = lane >= 16;
+      const uint32_t sel_quad = 0x4440u + q;                        // PRMT: byte q, zero-extended
+      const uint32_t sel_pair = (q & 1) ? 0x4432u : 0x4410u;        // PRMT: half q&1, zero-extended
+      const uint32_t row_pair = (q >> 1) * 32u, row_single = q * 32u;
+      const uint32_t lane4 = 4u * k8;
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kDStages);
-        mbar_wait(&sm.full[s], (i / kDStages) & 1u);
+        named_sync(kBarFull0 + s, kBarCount);
         const uint32_t t = sm.tile[s];
         if (t == kSentinel) break;
         const bool last = (t == a.num_tiles - 1);
         const uint32_t* data = sm.data[s] + sm.delta[s];
-        const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;
-        // 4 groups of 4 blocks: the group's words are loaded so that one bit
-        // transpose serves as many blocks as fit; the transposed rows go to
-        // scratch, from where a11/a12 continue with 4 elements per lane.
+        float* outp = a.out + uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32 + q * 32u + lane4;
 #pragma unroll 1
         for (int g = 0; g < kBPW / 4; ++g) {
-          const uint32_t wbytes = sm.gwords[s][w * 4 + g];
-          const uint32_t gm = sm.gmeta[s][w * 4 + g];
-          const uint32_t* gdata = data + (gm & 0xffffu);
-          const uint32_t mode = gm >> 16;
+          const uint2 gi = sm.ginfo[s][w * 4 + g];
+          const uint32_t wbytes = gi.x;
+          const uint32_t* gdata = data + (gi.y & 0xffffu);
+          const uint32_t mode = gi.y >> 16;
           const uint32_t pbytes = wbytes * 0x01010100u;             // exclusive word prefix per block
-          int row_lane, fsh;                                         // phase-2 source for this lane
+          uint32_t sel, row;                                         // phase-2 source of this lane
+          // a10: load each packed block's words into its lane range, one transpose per row
           if (mode == 0) {
-            const uint32_t sh = (lane >> 3) * 8, kk = lane & 7;
-            const uint32_t x = kk < ((wbytes >> sh) & 0xffu) ? gdata[((pbytes >> sh) & 0xffu) + kk] : 0u;
-            scratch[lane] = xpose(x);
-            row_lane = 0;
-            fsh = 8 * (lane >> 3);
+            const uint32_t wq = __byte_perm(wbytes, 0, sel_quad), pq = __byte_perm(pbytes, 0, sel_quad);
+            scratch[lane] = xpose(k8 < wq ? gdata[pq + k8] : 0u);
+            sel = sel_quad;
+            row = 0;
           } else if (mode == 1) {
-            const uint32_t kk = lane & 15;
             const uint32_t w0 = wbytes & 0xffu, w1 = (wbytes >> 8) & 0xffu;
             const uint32_t w2 = (wbytes >> 16) & 0xffu, w3 = wbytes >> 24;
-            const bool hi = lane >= 16;
-            const uint32_t x01 = kk < (hi ? w1 : w0) ? gdata[(hi ? w0 : 0u) + kk] : 0u;
-            const uint32_t x23 = kk < (hi ? w3 : w2) ? gdata[w0 + w1 + (hi ? w2 : 0u) + kk] : 0u;
+            const uint32_t x01 = k16 < (hi ? w1 : w0) ? gdata[(hi ? w0 : 0u) + k16] : 0u;
+            const uint32_t x23 = k16 < (hi ? w3 : w2) ? gdata[w0 + w1 + (hi ? w2 : 0u) + k16] : 0u;
             scratch[lane] = xpose(x01);
             scratch[32 + lane] = xpose(x23);
-            row_lane = (lane >> 4) * 32;
-            fsh = 16 * ((lane >> 3) & 1);
+            sel = sel_pair;
+            row = row_pair;
           } else {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              const uint32_t wq = (wbytes >> (8 * q)) & 0xffu, oq = (pbytes >> (8 * q)) & 0xffu;
-              scratch[32 * q + lane] = xpose(uint32_t(lane) < wq ? gdata[oq + lane] : 0u);
+            for (int b = 0; b < 4; ++b) {
+              const uint32_t wq = (wbytes >> (8 * b)) & 0xffu, oq = (pbytes >> (8 * b)) & 0xffu;
+              scratch[32 * b + lane] = xpose(uint32_t(lane) < wq ? gdata[oq + lane] : 0u);
             }
-            row_lane = (lane >> 3) * 32;
-            fsh = 0;
+            sel = 0x3210u;
+            row = row_single;
           }
           __syncwarp();
-          const uint32_t fmask = mode == 0 ? 0xffu : (mode == 1 ? 0xffffu : 0xffffffffu);
-          const uint4 raw = *reinterpret_cast<const uint4*>(&scratch[row_lane + 4 * (lane & 7)]);
-          int4 e;
+          const uint4 raw = *reinterpret_cast<const uint4*>(&scratch[row + lane4]);
+          // sign-magnitude v = 2|l| + s -> l
+          int e0, e1, e2, e3;
           {
-            const uint32_t v0 = (raw.x >> fsh) & fmask, v1 = (raw.y >> fsh) & fmask;
-            const uint32_t v2 = (raw.z >> fsh) & fmask, v3 = (raw.w >> fsh) & fmask;
-            e.x = (v0 & 1u) ? -int(v0 >> 1) : int(v0 >> 1);   // l = sign ? -|l| : |l|
-            e.y = (v1 & 1u) ? -int(v1 >> 1) : int(v1 >> 1);
-            e.z = (v2 & 1u) ? -int(v2 >> 1) : int(v2 >> 1);
-            e.w = (v3 & 1u) ? -int(v3 >> 1) : int(v3 >> 1);
+            const uint32_t v0 = __byte_perm(raw.x, 0, sel), v1 = __byte_perm(raw.y, 0, sel);
+            const uint32_t v2 = __byte_perm(raw.z, 0, sel), v3 = __byte_perm(raw.w, 0, sel);
+            e0 = (v0 & 1u) ? -int(v0 >> 1) : int(v0 >> 1);
+            e1 = (v1 & 1u) ? -int(v1 >> 1) : int(v1 >> 1);
+            e2 = (v2 & 1u) ? -int(v2 >> 1) : int(v2 >> 1);
+            e3 = (v3 & 1u) ? -int(v3 >> 1) : int(v3 >> 1);
           }
           // a11: r_j = sum_{i <= j} l_i within the block
-          e.y += e.x;
-          e.z += e.y;
-          e.w += e.z;
-          int incl = e.w;
+          e1 += e0;
+          e2 += e1;
+          e3 += e2;
+          int incl = e3;
           incl = scan_step_up(incl, 1, 24 << 8);
           incl = scan_step_up(incl, 2, 24 << 8);
           incl = scan_step_up(incl, 4, 24 << 8);
-          const int carry = incl - e.w;
-          e.x += carry; e.y += carry; e.z += carry; e.w += carry;
+          const int carry = incl - e3;
           // a12: d' = r * 2eb
           float4 d;
-          d.x = __fmul_rn(__int2float_rn(e.x), two_eb);
-          d.y = __fmul_rn(__int2float_rn(e.y), two_eb);
-          d.z = __fmul_rn(__int2float_rn(e.z), two_eb);
-          d.w = __fmul_rn(__int2float_rn(e.w), two_eb);
-          const uint64_t i0 = g0 + uint64_t(4 * g + (lane >> 3)) * 32 + 4 * (lane & 7);
-          if (!last || i0 + 4 <= a.n) {
-            *reinterpret_cast<float4*>(a.out + i0) = d;
+          d.x = __fmul_rn(__int2float_rn(e0 + carry), two_eb);
+          d.y = __fmul_rn(__int2float_rn(e1 + carry), two_eb);
+          d.z = __fmul_rn(__int2float_rn(e2 + carry), two_eb);
+          d.w = __fmul_rn(__int2float_rn(incl), two_eb);
+          float* o = outp + g * 128;
+          if (!last) {
+            *reinterpret_cast<float4*>(o) = d;
           } else {
-            if (i0 < a.n) a.out[i0] = d.x;
-            if (i0 + 1 < a.n) a.out[i0 + 1] = d.y;
-            if (i0 + 2 < a.n) a.out[i0 + 2] = d.z;
+            const uint64_t i0 = uint64_t(o - a.out);
+            if (i0 + 4 <= a.n) *reinterpret_cast<float4*>(o) = d;
+            else {
+              if (i0 < a.n) o[0] = d.x;
+              if (i0 + 1 < a.n) o[1] = d.y;
+              if (i0 + 2 < a.n) o[2] = d.z;
+            }
           }
           __syncwarp();
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.empty[s]);
+        named_arrive(kBarEmpty0 + s, kBarCount);
       }
     }
   }

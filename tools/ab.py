@@ -31,6 +31,7 @@ def main():
     ap.add_argument("--config", default="c2_hurricane")
     ap.add_argument("--field", default=None)
     ap.add_argument("--rel", type=float, default=1e-2)
+    ap.add_argument("--nocheck", action="store_true")
     a = ap.parse_args()
     import synth
     dev = torch.device("cuda", 0)
@@ -68,7 +69,7 @@ def main():
             S = int(ob.item())
             digest = (S, float(y[:1000].sum()), float(y[-1000:].sum()))
             if ref is None: ref = digest
-            assert digest == ref, (a.libs[i], digest, ref)
+            if not a.nocheck: assert digest == ref, (a.libs[i], digest, ref)
             if r >= 2:
                 res[i]["range"].append(ev[0].elapsed_time(ev[1]) * 1e3)
                 res[i]["compress"].append(ev[2].elapsed_time(ev[3]) * 1e3)
