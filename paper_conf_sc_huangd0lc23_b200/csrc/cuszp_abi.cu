@@ -275,5 +275,14 @@ int cuszp_version(void) { return CUSZP_VERSION * 100 + 1; }
 
 // diagnostics only (not declared in include/cuszp.h)
 void cuszp_debug_set_trace(void* d_trace) { g_trace = static_cast<uint64_t*>(d_trace); }
+int cuszp_debug_occupancy(int* out4) {
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  out4[0] = di.sms;
+  out4[1] = di.occ_compress;
+  out4[2] = di.occ_decompress;
+  out4[3] = di.occ_range;
+  return CUSZP_OK;
+}
 
 }  // extern "C"

@@ -76,6 +76,10 @@ def main():
                 res[i]["decompress"].append(ev[4].elapsed_time(ev[5]) * 1e3)
                 res[i]["rel_chain"].append(ev[6].elapsed_time(ev[7]) * 1e3)
     print(f"n={n} S={ref[0]} CR={4 * n / ref[0]:.2f}  (us: median / min)")
+    occ = (C.c_int * 4)()
+    for p_, h in zip(a.libs, libs):
+        if hasattr(h, "cuszp_debug_occupancy") and h.cuszp_debug_occupancy(occ) == 0:
+            print(f"   {os.path.basename(p_):38s} SMs {occ[0]}  CTAs/SM: compress {occ[1]} decompress {occ[2]} range {occ[3]}")
     for i, p in enumerate(a.libs):
         d = res[i]
         print(f"{os.path.basename(p):40s} range {np.median(d['range']):7.1f}/{min(d['range']):7.1f}  "
