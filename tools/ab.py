@@ -32,6 +32,7 @@ def main():
     ap.add_argument("--field", default=None)
     ap.add_argument("--rel", type=float, default=1e-2)
     ap.add_argument("--nocheck", action="store_true")
+    ap.add_argument("--dirty-flush", action="store_true")
     a = ap.parse_args()
     import synth
     dev = torch.device("cuda", 0)
@@ -45,7 +46,19 @@ def main():
     ob = torch.zeros(1, dtype=torch.int64, device=dev)
     mm = torch.empty(2, dtype=torch.float32, device=dev)
     y = torch.empty(n, dtype=torch.float32, device=dev)
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    flush_buf = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    sink = torch.empty(1, dtype=torch.int64, device=dev)
+
+    class _F:
+        @staticmethod
+        def zero_():
+            # write then read 512 MB: L2 ends up holding CLEAN lines of an
+            # unrelated buffer (a write-only flush leaves ~126 MB of dirty lines
+            # whose write-back would be charged to the next timed kernel)
+            flush_buf.zero_()
+            if not a.dirty_flush:
+                sink.copy_(flush_buf.view(torch.int64).sum())
+    flush = _F
     sp = torch.cuda.current_stream().cuda_stream
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(9)]
     res = {i: {"range": [], "compress": [], "decompress": [], "rel_chain": []} for i in range(len(libs))}

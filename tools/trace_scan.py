@@ -5,8 +5,8 @@
 Installs a trace buffer (cuszp_debug_set_trace), runs range + compress +
 decompress on one field and prints, per kernel, the distribution of the
 per-tile phases recorded with %globaltimer:
-  slot 0 ticket taken, 1 data in shared memory, 2 aggregate published,
-  3 look-back start, 4 prefix resolved, 5 windows walked, 6 spins, 7 smid<<32|cta
+  slot 0 ticket taken, 1 compute start, 2 aggregate published,
+  3 look-back start, 4 prefix resolved, 5 windows walked, 6 spins, 7 data in shared memory
 """
 from __future__ import annotations
 
@@ -49,7 +49,8 @@ def report(name, tr, total_ns):
     pfx = (tr[:, 4] - t0) / 1e3
     print(f"== {name}: {tr.shape[0]} tiles, kernel span {total_ns / 1e3:.1f} us (first ticket .. last prefix "
           f"{(tr[:, 4].max() - t0) / 1e3:.1f} us)")
-    print(f"  ticket -> data landed   (us) {pct(landed - ticket)}")
+    print(f"  ticket -> data landed   (us) {pct((tr[:, 7] - t0) / 1e3 - ticket)}")
+    print(f"  landed -> compute start (us) {pct(landed - (tr[:, 7] - t0) / 1e3)}  (waiting for a writer's meta slot)")
     print(f"  landed -> aggregate     (us) {pct(agg - landed)}")
     print(f"  aggregate -> lb start   (us) {pct(lb0 - agg)}")
     print(f"  look-back duration      (us) {pct(pfx - lb0)}")
@@ -81,12 +82,13 @@ def main():
     ap.add_argument("--lib", default=os.path.join(ROOT, "paper_conf_sc_huangd0lc23_b200", "libcuszp.so"))
     ap.add_argument("--config", default="c2_hurricane")
     ap.add_argument("--rel", type=float, default=1e-2)
+    ap.add_argument("--field", default=None)
     a = ap.parse_args()
     import synth
 
     h = load(a.lib)
     dev = torch.device("cuda", 0)
-    x = synth.field_for_config(a.config, device=dev)
+    x = synth.field_for_config(a.config, device=dev, field=a.field)
     n = x.numel()
     nt = ((n + 31) // 32 + 127) // 128
     ws = torch.zeros(h.cuszp_workspace_bytes(n), dtype=torch.uint8, device=dev)
