@@ -218,7 +218,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t j = uint32_t(warp - 1);; j += kWriters) {
         const int m = int(j % kMeta);
         const uint32_t par = (j / kMeta) & 1u;
+#ifdef CUSZP_C_POLL
         while (!mbar_test(&sm.staged[m], par)) __nanosleep(4 * CUSZP_C_POLL_NS);
+#else
+        mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
+#endif
         const TileMeta& md = sm.meta[m];
         const uint32_t t = md.tile;
         if (t == kSentinel) break;
@@ -269,7 +273,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
+#ifdef CUSZP_C_POLL
         while (!mbar_test(&sm.full[s], (i / kStages) & 1u)) __nanosleep(CUSZP_C_POLL_NS);
+#else
+        mbar_wait(&sm.full[s], (i / kStages) & 1u);         // suspending wait: no issue slots taken
+#endif
         const uint32_t t = sm.in_tile[s];
         if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
         // meta slot m free (tile i - kMeta released)
@@ -296,7 +304,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         // blocks per transpose), and a ballot of the non-zero words gives every
         // block's word count (the top plane is non-zero by definition of F).
 #pragma unroll
+#ifdef CUSZP_DIAG_NOWORK
+        for (int g = 0; g < 0; ++g) {   // diagnostics only: pipeline without the encode work
+#else
         for (int g = 0; g < kBPW / 4; ++g) {
+#endif
           float x[4];
 #pragma unroll
           for (int q = 0; q < 4; ++q) {

@@ -33,6 +33,10 @@ namespace {
 #define CUSZP_D_STAGES 4
 #endif
 constexpr int kDStages = CUSZP_D_STAGES;
+#ifndef CUSZP_D_UNROLL
+#define CUSZP_D_UNROLL 4
+#endif
+constexpr int kDUnroll = CUSZP_D_UNROLL;                        // decode groups interleaved per iteration
 constexpr int kChunkTiles = 4;                                  // tiles per look-back unit
 constexpr int kGroups = kTileBlocks / 4;                        // 32 decode groups per tile
 constexpr int kDataWords = kTileBlocks * kMaxBlockWords + 8;   // 3208 words: worst tile + alignment slack
@@ -59,7 +63,7 @@ struct DecompressSmem {
 };
 
 // named barriers (id 0 is __syncthreads)
-constexpr uint32_t kBarFull0 = 1, kBarEmpty0 = kBarFull0 + kDStages;
+constexpr uint32_t kBarEmpty0 = 1;
 constexpr uint32_t kBarReady0 = kBarEmpty0 + kDStages, kBarFree0 = kBarReady0 + 2;
 constexpr uint32_t kBarCount = 32 + 32 * kComputeWarps;   // loader + compute warps
 static_assert(kBarFree0 + 2 <= 16, "named barriers");
@@ -195,28 +199,21 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     } else if (warp == 1) {
       // -------------------------------------------------------------- loader
       // Tile k goes to stage k % S once the compute warps released it (named
-      // barrier EMPTY); one step behind, the loader waits for tile k-1's TMA
-      // bytes and signals the compute warps (named barrier FULL).
+      // barrier EMPTY); the compute warps wait for its bytes on the stage's
+      // mbarrier themselves (suspending try_wait), so up to S payload copies
+      // are in flight and the loader never waits for a TMA to land.
       uint32_t k = 0;              // tiles loaded so far
-      bool prev_pending = false;   // tile k-1 loaded, not yet signalled
-      auto signal_prev = [&]() {
-        if (prev_pending) {
-          const int sp = int((k - 1) % kDStages);
-          mbar_wait(&sm.full[sp], ((k - 1) / kDStages) & 1u);
-          named_arrive(kBarFull0 + sp, kBarCount);
-          prev_pending = false;
-        }
-      };
       for (uint32_t i = 0;; ++i) {
         const int b = int(i & 1u);
         named_sync(kBarReady0 + b, 64);
         const ChunkDesc& cd = sm.chunk[b];
         if (cd.chunk == kSentinel) {
-          signal_prev();
           const int s = int(k % kDStages);
           if (k >= uint32_t(kDStages)) named_sync(kBarEmpty0 + s, kBarCount);
-          if (lane == 0) sm.tile[s] = kSentinel;
-          named_arrive(kBarFull0 + s, kBarCount);
+          if (lane == 0) {
+            sm.tile[s] = kSentinel;
+            mbar_arrive(&sm.full[s]);
+          }
           break;
         }
         for (uint32_t j = 0; j < cd.ntiles; ++j) {
@@ -245,8 +242,6 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             mbar_arrive_expect_tx(&sm.full[s], tma_bytes);   // one phase per use, even with 0 bytes
             if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
           }
-          signal_prev();
-          prev_pending = true;
           ++k;
         }
         named_arrive(kBarFree0 + b, 64);
@@ -266,14 +261,18 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
       const uint32_t lane4 = 4u * k8;
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kDStages);
-        named_sync(kBarFull0 + s, kBarCount);
+        mbar_wait(&sm.full[s], (i / kDStages) & 1u);          // tile's payload landed (suspending wait)
         const uint32_t t = sm.tile[s];
         if (t == kSentinel) break;
         const bool last = (t == a.num_tiles - 1);
         const uint32_t* data = sm.data[s] + sm.delta[s];
         float* outp = a.out + uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32 + q * 32u + lane4;
-#pragma unroll 1
+#pragma unroll kDUnroll
+#ifdef CUSZP_DIAG_NOWORK
+        for (int g = 0; g < 0; ++g) {   // diagnostics only: pipeline without the decode work
+#else
         for (int g = 0; g < kBPW / 4; ++g) {
+#endif
           const uint2 gi = sm.ginfo[s][w * 4 + g];
           const uint32_t wbytes = gi.x;
           const uint32_t* gdata = data + (gi.y & 0xffffu);
