@@ -52,6 +52,8 @@ constexpr int kWriters = CUSZP_C_WRITERS;        // scan + writer warps
 constexpr int kMeta = CUSZP_C_META;              // tiles between "computed" and "released"
 constexpr uint32_t kRing = CUSZP_C_RING_WORDS;   // words per compute-warp ring (power of 2)
 constexpr int kFirstCompute = 1 + kWriters;
+constexpr int kTix = 16;                          // ticket ring: producer -> writers (early look-back)
+static_assert(kStages + kMeta + kWriters <= kTix, "ticket ring");
 constexpr int kCThreads = (kFirstCompute + kComputeWarps) * 32;
 static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * kMaxBlockWords, "ring size");
 
@@ -70,7 +72,8 @@ struct CompressSmem {
   uint32_t meta_done[kMeta];
   uint32_t tail[kComputeWarps];                  // ring words released (monotonic)
   uint32_t released;                             // CTA-local tiles released (monotonic)
-  uint64_t full[kStages], empty[kStages], staged[kMeta];
+  uint32_t tix[kTix];                            // tile of CTA-local tile j (slot j % kTix)
+  uint64_t full[kStages], empty[kStages], staged[kMeta], tixbar[kTix];
 };
 
 __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
@@ -153,7 +156,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   extern __shared__ __align__(128) unsigned char smem_raw[];
   CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
-  const int warp = threadIdx.x >> 5;
+  const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);   // provably warp-uniform (no divergence checks before warp-sync ops)
   const uint32_t epoch = running_epoch(a.ws);
 
   // ---- eb_abs (Eq 1): ABS -> delta; REL -> lambda * (max - min) over the (min,max) pairs
@@ -181,6 +184,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kComputeWarps); }
     for (int m = 0; m < kMeta; ++m) { mbar_init(&sm.staged[m], 1); sm.meta_done[m] = 0; }
+    for (int k = 0; k < kTix; ++k) mbar_init(&sm.tixbar[k], 1);
     for (int w = 0; w < kComputeWarps; ++w) sm.tail[w] = 0;
     sm.released = 0;
     fence_mbar_init();
@@ -191,17 +195,25 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
     if (warp == 0) {
       // ------------------------------------------------------------ producer
       if (lane == 0) {
-        uint32_t next = atomicAdd(&a.ws->ticket, 1u);   // tickets are prefetched one ahead
         for (uint32_t i = 0;; ++i) {
           const int s = int(i % kStages);
           mbar_wait(&sm.empty[s], ((i / kStages) & 1u) ^ 1u);
-          const uint32_t t = next;
+          // ticket taken only once the stage is free: a prefetched ticket would
+          // wait a whole tile of compute before its load, and every later tile's
+          // look-back would wait for it
+          const uint32_t t = atomicAdd(&a.ws->ticket, 1u);
           if (t >= a.num_tiles) {
             sm.in_tile[s] = kSentinel;
             mbar_arrive(&sm.full[s]);
+            // every writer must see a sentinel: one in each of the next kWriters ticket slots
+            for (uint32_t k = 0; k < uint32_t(kWriters); ++k) {
+              sm.tix[(i + k) % kTix] = kSentinel;
+              mbar_arrive(&sm.tixbar[(i + k) % kTix]);
+            }
             break;
           }
-          next = atomicAdd(&a.ws->ticket, 1u);
+          sm.tix[i % kTix] = t;                          // writers start the look-back now
+          mbar_arrive(&sm.tixbar[i % kTix]);
           trace_put(a.trace, t, 0, global_ns());
           sm.in_tile[s] = t;
           const uint64_t e0 = uint64_t(t) * kTileElems;
@@ -218,15 +230,19 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t j = uint32_t(warp - 1);; j += kWriters) {
         const int m = int(j % kMeta);
         const uint32_t par = (j / kMeta) & 1u;
-#ifdef CUSZP_C_POLL
-        while (!mbar_test(&sm.staged[m], par)) __nanosleep(4 * CUSZP_C_POLL_NS);
-#else
-        mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
-#endif
-        const TileMeta& md = sm.meta[m];
-        const uint32_t t = md.tile;
+        // the tile's ticket is known as soon as its load is issued: resolve its
+        // exclusive prefix (the look-back needs only the predecessors' words)
+        // while the tile is still loading and being encoded
+        mbar_wait(&sm.tixbar[j % kTix], (j / kTix) & 1u);
+        const uint32_t t = sm.tix[j % kTix];
         if (t == kSentinel) break;
+        uint32_t nw = 0, ns = 0;
+        const uint64_t t_lb = a.trace ? global_ns() : 0;
+        const uint64_t excl = resolve_excl(a.status, t, epoch, &nw, &ns);
+        mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
+        const TileMeta& md = sm.meta[m];
         const uint32_t agg = md.agg;
+        if (lane == 0 && t > 0) publish_prefix(a.status, t, excl + agg, epoch);
         const uint32_t cnt = lane < kComputeWarps ? md.cnt[lane] : 0u;
         const uint32_t hd = lane < kComputeWarps ? md.head[lane] : 0u;
         uint32_t incl = cnt;
@@ -235,9 +251,6 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           const uint32_t y = __shfl_up_sync(kFull, incl, o);
           if (lane >= o) incl += y;
         }
-        uint32_t nw = 0, ns = 0;
-        const uint64_t t_lb = a.trace ? global_ns() : 0;
-        const uint64_t excl = resolve_prefix(a.status, t, agg, epoch, &nw, &ns);
         if (lane == 0 && a.trace) {
           trace_put(a.trace, t, 3, t_lb);
           trace_put(a.trace, t, 4, global_ns());
@@ -279,20 +292,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         mbar_wait(&sm.full[s], (i / kStages) & 1u);         // suspending wait: no issue slots taken
 #endif
         const uint32_t t = sm.in_tile[s];
-        if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
+        if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 7, global_ns());
         // meta slot m free (tile i - kMeta released)
         while (int(i - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(CUSZP_C_POLL_NS);
-        if (t == kSentinel) {
-          // every writer must see a sentinel: post one in each of the next kWriters slots
-          if (w == 0 && lane == 0) {
-            for (uint32_t k = 0; k < uint32_t(kWriters); ++k) {
-              while (int(i + k - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(64);
-              sm.meta[(i + k) % kMeta].tile = kSentinel;
-              mbar_arrive(&sm.staged[(i + k) % kMeta]);
-            }
-          }
-          break;
-        }
+        if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
+        if (t == kSentinel) break;                    // the writers stop on the ticket ring
         const bool last = (t == a.num_tiles - 1);
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;   // first element of the warp
         const float* src = &sm.in[s][w * kBPW * 32];

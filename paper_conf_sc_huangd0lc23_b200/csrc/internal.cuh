@@ -256,9 +256,11 @@ __device__ __forceinline__ void publish_aggregate(uint64_t* status, uint32_t t, 
 #ifndef CUSZP_LB_BACKOFF_MAX
 #define CUSZP_LB_BACKOFF_MAX 1024
 #endif
-__device__ __forceinline__ uint64_t resolve_prefix(uint64_t* status, uint32_t t, uint64_t agg,
-                                                   uint32_t epoch, uint32_t* n_windows = nullptr,
-                                                   uint32_t* n_spins = nullptr) {
+// resolve_excl: the look-back proper (all 32 lanes): tile t's exclusive
+// prefix, without publishing anything.  It needs only the predecessors'
+// words, so it may run before tile t's own aggregate is known.
+__device__ __forceinline__ uint64_t resolve_excl(const uint64_t* status, uint32_t t, uint32_t epoch,
+                                                 uint32_t* n_windows = nullptr, uint32_t* n_spins = nullptr) {
   if (t == 0) return 0;
   constexpr int K = CUSZP_LB_K;
   uint32_t windows = 0, spins = 0;
@@ -299,9 +301,22 @@ __device__ __forceinline__ uint64_t resolve_prefix(uint64_t* status, uint32_t t,
     if (pmask) break;
     top -= 32 * K;
   }
-  if (lane == 0) st_relaxed_u64(status + t, tag | kPrefixFlag | (excl + agg));
   if (n_windows) *n_windows = windows;
   if (n_spins) *n_spins = spins;
+  return excl;
+}
+
+// publish_prefix: one thread; tile t's inclusive prefix.
+__device__ __forceinline__ void publish_prefix(uint64_t* status, uint32_t t, uint64_t incl, uint32_t epoch) {
+  st_relaxed_u64(status + t, (uint64_t(epoch) << kEpochShift) | kPrefixFlag | incl);
+}
+
+__device__ __forceinline__ uint64_t resolve_prefix(uint64_t* status, uint32_t t, uint64_t agg,
+                                                   uint32_t epoch, uint32_t* n_windows = nullptr,
+                                                   uint32_t* n_spins = nullptr) {
+  if (t == 0) return 0;
+  const uint64_t excl = resolve_excl(status, t, epoch, n_windows, n_spins);
+  if ((threadIdx.x & 31) == 0) publish_prefix(status, t, excl + agg, epoch);
   return excl;
 }
 

@@ -49,8 +49,8 @@ def report(name, tr, total_ns):
     pfx = (tr[:, 4] - t0) / 1e3
     print(f"== {name}: {tr.shape[0]} tiles, kernel span {total_ns / 1e3:.1f} us (first ticket .. last prefix "
           f"{(tr[:, 4].max() - t0) / 1e3:.1f} us)")
-    print(f"  ticket -> data landed   (us) {pct((tr[:, 7] - t0) / 1e3 - ticket)}")
-    print(f"  landed -> compute start (us) {pct(landed - (tr[:, 7] - t0) / 1e3)}  (waiting for a writer's meta slot)")
+    print(f"  TMA issue -> landed     (us) {pct((tr[:, 7] - t0) / 1e3 - ticket)}")
+    print(f"  landed -> compute start (us) {pct(landed - (tr[:, 7] - t0) / 1e3)}  (meta-slot wait)")
     print(f"  landed -> aggregate     (us) {pct(agg - landed)}")
     print(f"  aggregate -> lb start   (us) {pct(lb0 - agg)}")
     print(f"  look-back duration      (us) {pct(pfx - lb0)}")
