@@ -288,14 +288,34 @@ def run_ours(args, rank, world, dev):
     if world > 1:
         torch.distributed.barrier()
 
-    # correctness spot check of the last round trip (device-side, bound of DESIGN sec 5)
-    f_last, rel_last = jobs[-1]
-    hdr = cz.read_header(out)
-    assert hdr["status"] == 0 and cz.last_status(ws) == cz.OK
-    xl = xs[f_last]
-    err = (y[: xl.numel()].double() - xl.double()).abs().max().item()
-    ulp_max = float(np.spacing(np.float32(xl.abs().max().item())))
-    assert err <= hdr["eb_abs"] + ulp_max, (err, hdr["eb_abs"])
+    # verification of every round trip on the device with the fused quality
+    # kernel (cuszp_quality; untimed): the bound of
+    # DESIGN sec 5, PSNR per job, and the quality kernel's own HBM rate
+    quality = {"psnr": {}, "max_abs_err_over_eb": {}}
+    qev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    q_ms = []
+    for f, rel in jobs:
+        x = xs[f]
+        n = n_of[f]
+        cz.check(lib.cuszp_range(x.data_ptr(), n, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
+        cz.check(lib.cuszp_compress_minmax(x.data_ptr(), n, float(rel), mm_local.data_ptr(), 1, out.data_ptr(),
+                                           cap, out_bytes.data_ptr(), ws.ptr(), ws.nbytes, sp), "compress")
+        cz.check(lib.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.ptr(), ws.nbytes, sp), "decompress")
+        hdr = cz.read_header(out)
+        assert hdr["status"] == 0 and cz.last_status(ws) == cz.OK
+        flush_l2()
+        qev[0].record(stream)
+        qraw = cz.quality(x, y[:n], bound=float(hdr["eb_abs"]), sync=False)
+        qev[1].record(stream)
+        torch.cuda.synchronize(dev)
+        q_ms.append(qev[0].elapsed_time(qev[1]))
+        qv = qraw.cpu()
+        ulp_max = float(np.spacing(np.float32(max(abs(qv[0].item()), abs(qv[1].item())))))
+        assert qv[3].item() <= hdr["eb_abs"] + ulp_max, (f, rel, qv[3].item(), hdr["eb_abs"])
+        quality["psnr"][f"{f}@{rel:g}"] = round(qv[7].item(), 3)
+        quality["max_abs_err_over_eb"][f"{f}@{rel:g}"] = round(qv[3].item() / hdr["eb_abs"], 6)
+    q_bytes = sum(8 * n_of[f] for f, _ in jobs)
+    quality["kernel_gbs"] = q_bytes / (sum(q_ms) / 1e3) / 1e9
 
     t_dev = torch.tensor([acc["range"], acc["compress"], acc["decompress"]], dtype=torch.float64, device=dev)
     if world > 1:
@@ -343,6 +363,8 @@ def run_ours(args, rank, world, dev):
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
         "gpu_launches": 3 * len(jobs) * K,
+        "quality": dict(quality, frac_of_peak=quality["kernel_gbs"] / peak,
+                        kernel="cuszp_quality (fused compareData statistics, untimed verification pass)"),
         "clocks": clk,
         "wall_s_timed_region": t_wall,
         "paper_context": PAPER_A100,

@@ -137,6 +137,40 @@ int cuszp_decompress_host(const void* h_in, size_t in_bytes, float* h_out, size_
                           void* d_in_scratch, float* d_out_scratch,
                           void* d_ws, size_t ws_bytes, void* stream);
 
+/* ---- reconstruction quality on the device ----
+ * The statistics the paper's artifact reads off QCAT compareData
+ * (P:1918-1933), PSNR as in sec 2.1, all in fp64.  x = original,
+ * y = reconstruction, e_i = x_i - y_i (exact in fp64):
+ *   min, max, range = max - min of x;
+ *   max_abs_err = max |e_i|;  max_rel_err = max_abs_err / range;
+ *   max_pw_rel_err = max over x_i != 0 of |e_i| / |x_i|;
+ *   mse = sum e_i^2 / n;  psnr = 20 log10(range) - 10 log10(mse);
+ *   nrmse = sqrt(mse) / range;  norm_err = sqrt(sum e_i^2);
+ *   norm_err_norm = norm_err / sqrt(sum x_i^2);
+ *   pearson = sum (x-mx)(y-my) / sqrt(sum (x-mx)^2 sum (y-my)^2);
+ *   n_over_bound = #{i : |e_i| > bound}  (pass the eb_abs of the stream).
+ * Degenerate inputs follow IEEE (range 0 -> inf/NaN ratios; mse 0 -> psnr
+ * +inf).  Inputs are expected finite. */
+typedef struct cuszp_quality_stats {
+  double min, max, range;
+  double max_abs_err, max_rel_err, max_pw_rel_err;
+  double mse, psnr, nrmse;
+  double norm_err, norm_err_norm, pearson;
+  unsigned long long n, n_over_bound;
+} cuszp_quality_stats;
+
+/* Workspace of cuszp_quality (independent of n); caller-zeroed once,
+ * left zeroed by every call. */
+size_t cuszp_quality_workspace_bytes(void);
+
+/* One kernel, one pass over d_x and d_y (8n bytes), writes *d_q (device
+ * memory, 8-byte aligned) stream-ordered.  Sums are folded in a fixed
+ * order: the result is deterministic for a given device.
+ * Sync errors: EINVAL (NULL pointers, n = 0, misaligned pointers, NaN
+ * bound), ENOSPACE (ws_bytes too small), ECUDA. */
+int cuszp_quality(const float* d_x, const float* d_y, size_t n, double bound,
+                  cuszp_quality_stats* d_q, void* d_ws, size_t ws_bytes, void* stream);
+
 /* Human-readable status name. */
 const char* cuszp_status_string(int status);
 

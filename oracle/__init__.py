@@ -70,6 +70,7 @@ def lib():
             h.oracle_compress_minmax.restype = i32
             h.oracle_decompress.argtypes = [vp, u64, vp, u64]
             h.oracle_decompress.restype = i32
+            h.oracle_quality.argtypes = [vp, vp, u64, C.c_double, vp, vp]
             _lib = h
     return _lib
 
@@ -166,3 +167,19 @@ def decompress(stream, n: int) -> tuple[int, np.ndarray]:
     out = np.zeros(int(n), np.float32)
     st = lib().oracle_decompress(_ptr(s), s.size, _ptr(out), int(n))
     return st, out
+
+
+QUALITY_KEYS = ("min", "max", "range", "max_abs_err", "max_rel_err", "max_pw_rel_err", "mse", "psnr", "nrmse",
+                "norm_err", "norm_err_norm", "pearson")
+
+
+def quality(x, y, bound: float = -1.0) -> dict:
+    """Reconstruction statistics of QCAT compareData in fp64."""
+    xa, ya = _f32(x), _f32(y)
+    assert xa.size == ya.size and xa.size > 0
+    out = np.zeros(12, np.float64)
+    cnt = np.zeros(2, np.uint64)
+    lib().oracle_quality(_ptr(xa), _ptr(ya), xa.size, float(bound), _ptr(out), _ptr(cnt))
+    d = dict(zip(QUALITY_KEYS, (float(v) for v in out)))
+    d["n"], d["n_over_bound"] = int(cnt[0]), int(cnt[1])
+    return d

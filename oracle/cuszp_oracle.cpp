@@ -321,4 +321,60 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
   return ORACLE_OK;
 }
 
+/* Reconstruction quality, each statistic written out by its definition
+ * (DESIGN.md sec 10): the printed artifact values of P:1918-1933 satisfy
+ * exactly these relations (tests/test_oracle_quality.py pins them). */
+void oracle_quality(const float* x, const float* y, uint64_t n, double bound, double out[12],
+                    uint64_t out_counts[2]) {
+  /* value range of the original (Min, Max, range) */
+  double mn = x[0], mx = x[0];
+  for (uint64_t i = 1; i < n; ++i) {
+    if (x[i] < mn) mn = x[i];
+    if (x[i] > mx) mx = x[i];
+  }
+  const double range = mx - mn;
+  /* pass 1: means of x and y */
+  double sum_x = 0.0, sum_y = 0.0;
+  for (uint64_t i = 0; i < n; ++i) {
+    sum_x += double(x[i]);
+    sum_y += double(y[i]);
+  }
+  const double mean_x = sum_x / double(n), mean_y = sum_y / double(n);
+  /* pass 2: errors and centred sums */
+  double max_abs = 0.0, max_pw = 0.0, sum_e2 = 0.0, sum_x2 = 0.0;
+  double cxx = 0.0, cyy = 0.0, cxy = 0.0;
+  uint64_t over = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    const double e = double(x[i]) - double(y[i]);
+    const double ae = e < 0 ? -e : e;
+    if (ae > max_abs) max_abs = ae;                        /* Max absolute error */
+    if (x[i] != 0.0f) {                                    /* Max pw relative error */
+      const double ax = x[i] < 0 ? -double(x[i]) : double(x[i]);
+      if (ae / ax > max_pw) max_pw = ae / ax;
+    }
+    if (ae > bound) ++over;
+    sum_e2 += e * e;
+    sum_x2 += double(x[i]) * double(x[i]);
+    const double dx = double(x[i]) - mean_x, dy = double(y[i]) - mean_y;
+    cxx += dx * dx;
+    cyy += dy * dy;
+    cxy += dx * dy;
+  }
+  const double mse = sum_e2 / double(n);
+  out[0] = mn;
+  out[1] = mx;
+  out[2] = range;
+  out[3] = max_abs;
+  out[4] = max_abs / range;                                /* Max relative error */
+  out[5] = max_pw;
+  out[6] = mse;
+  out[7] = 20.0 * std::log10(range) - 10.0 * std::log10(mse);   /* PSNR (dB) */
+  out[8] = std::sqrt(mse) / range;                         /* NRMSE */
+  out[9] = std::sqrt(sum_e2);                              /* normErr */
+  out[10] = std::sqrt(sum_e2) / std::sqrt(sum_x2);         /* normErr_norm */
+  out[11] = cxy / std::sqrt(cxx * cyy);                    /* pearson coeff */
+  out_counts[0] = n;
+  out_counts[1] = over;
+}
+
 }  // extern "C"

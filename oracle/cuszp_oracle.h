@@ -93,6 +93,16 @@ int oracle_compress_minmax(const float* x, uint64_t n, float lambda,
 int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out,
                       uint64_t n);
 
+/* ---- reconstruction quality -------------------
+ * The statistics of the paper's artifact output (QCAT compareData,
+ * P:1918-1933) and PSNR (sec 2.1), in fp64, two plain passes
+ * (means first, then centred sums).  out[0..11] = min, max, range,
+ * max_abs_err, max_rel_err, max_pw_rel_err, mse, psnr, nrmse, norm_err,
+ * norm_err_norm, pearson; out_counts[0..1] = n, #{|x_i - y_i| > bound}.
+ * n must be > 0. */
+void oracle_quality(const float* x, const float* y, uint64_t n, double bound,
+                    double out[12], uint64_t out_counts[2]);
+
 #ifdef __cplusplus
 }
 #endif

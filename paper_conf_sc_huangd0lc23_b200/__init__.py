@@ -28,7 +28,7 @@ BLOCK_LEN = 32
 __all__ = [
     "ABS", "REL", "Workspace", "compress", "compress_minmax", "decompress", "value_range",
     "max_compressed_bytes", "workspace_bytes", "last_status", "read_header", "compress_host",
-    "decompress_host", "CuszpError", "exact_bytes_from_F",
+    "decompress_host", "CuszpError", "exact_bytes_from_F", "quality", "QUALITY_KEYS",
 ]
 
 
@@ -205,3 +205,36 @@ def decompress_host(h_in, in_bytes: int, h_out, d_in_scratch: torch.Tensor, d_ou
     check(lib().cuszp_decompress_host(pin, int(in_bytes), pout, n, d_in_scratch.data_ptr(),
                                       d_out_scratch.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
           "cuszp_decompress_host")
+
+
+QUALITY_KEYS = ("min", "max", "range", "max_abs_err", "max_rel_err", "max_pw_rel_err", "mse", "psnr", "nrmse",
+                "norm_err", "norm_err_norm", "pearson")
+_qws_cache: dict = {}
+
+
+def quality(x: torch.Tensor, y: torch.Tensor, bound: float = -1.0, out: torch.Tensor | None = None,
+            stream=None, sync: bool = True):
+    """Reconstruction statistics (QCAT compareData's) of y
+    against x in one fused device pass (cuszp_quality).  ``out`` (float64
+    CUDA tensor of 14) receives the raw cuszp_quality_stats; with sync=True
+    the statistics are returned as a dict (one 112-byte device->host copy)."""
+    _require_cuda(x, "x", torch.float32)
+    _require_cuda(y, "y", torch.float32)
+    if x.numel() != y.numel():
+        raise ValueError("x and y must have the same number of elements")
+    key = (x.device.index, torch.cuda.current_stream(x.device).cuda_stream)
+    qws = _qws_cache.get(key)
+    if qws is None:
+        qws = torch.zeros(int(lib().cuszp_quality_workspace_bytes()), dtype=torch.uint8, device=x.device)
+        _qws_cache[key] = qws
+    if out is None:
+        out = torch.empty(14, dtype=torch.float64, device=x.device)
+    check(lib().cuszp_quality(x.data_ptr(), y.data_ptr(), x.numel(), float(bound), out.data_ptr(), qws.data_ptr(),
+                              qws.numel(), _stream_ptr(stream)), "cuszp_quality")
+    if not sync:
+        return out
+    raw = out.cpu()
+    d = dict(zip(QUALITY_KEYS, (float(v) for v in raw[:12])))
+    cnt = raw[12:].view(torch.int64)
+    d["n"], d["n_over_bound"] = int(cnt[0]), int(cnt[1])
+    return d

@@ -22,7 +22,7 @@ SYMBOLS = (
     "cuszp_max_compressed_bytes", "cuszp_compressed_bytes_from_F", "cuszp_workspace_bytes",
     "cuszp_range", "cuszp_compress", "cuszp_compress_minmax", "cuszp_decompress",
     "cuszp_last_status", "cuszp_read_header", "cuszp_compress_host", "cuszp_decompress_host",
-    "cuszp_status_string", "cuszp_version",
+    "cuszp_status_string", "cuszp_version", "cuszp_quality_workspace_bytes", "cuszp_quality",
 )
 
 _lock = threading.Lock()
@@ -61,6 +61,10 @@ def _declare(h):
     h.cuszp_decompress_host.restype = i32
     h.cuszp_status_string.argtypes = [i32]
     h.cuszp_status_string.restype = C.c_char_p
+    h.cuszp_quality_workspace_bytes.argtypes = []
+    h.cuszp_quality_workspace_bytes.restype = sz
+    h.cuszp_quality.argtypes = [vp, vp, sz, C.c_double, vp, vp, sz, vp]
+    h.cuszp_quality.restype = i32
     h.cuszp_version.argtypes = []
     h.cuszp_version.restype = i32
 

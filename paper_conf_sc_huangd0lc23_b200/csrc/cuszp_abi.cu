@@ -16,7 +16,7 @@ uint64_t num_tiles(uint64_t n) { return (num_blocks(n) + kTileBlocks - 1) / kTil
 
 struct DeviceInfo {
   int sms = 0;
-  int occ_compress = 0, occ_decompress = 0, occ_range = 0;
+  int occ_compress = 0, occ_decompress = 0, occ_range = 0, occ_quality = 0;
 };
 
 // Per-device launch geometry, computed once: persistent grids of
@@ -38,7 +38,8 @@ int device_info(DeviceInfo* out) {
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_compress, compress_kernel, compress_threads(), cs) != cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_decompress, decompress_kernel, decompress_threads(), ds) !=
             cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess)
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_quality, quality_kernel, 256, 0) != cudaSuccess)
       return CUSZP_ECUDA;
     cache[dev] = d;
     have[dev] = true;
@@ -124,6 +125,28 @@ int cuszp_range(const float* d_in, size_t n, float* d_minmax, void* d_ws, size_t
   if (grid > want) grid = want;
   if (grid < 1) grid = 1;
   range_kernel<<<unsigned(grid), 256, 0, static_cast<cudaStream_t>(stream)>>>(a);
+  return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+}
+
+size_t cuszp_quality_workspace_bytes(void) { return 128 + 128 * size_t(kQualityMaxGrid); }
+
+int cuszp_quality(const float* d_x, const float* d_y, size_t n, double bound, cuszp_quality_stats* d_q, void* d_ws,
+                  size_t ws_bytes, void* stream) {
+  static_assert(sizeof(cuszp_quality_stats) == 14 * 8, "cuszp_quality_stats layout");
+  if (d_x == nullptr || d_y == nullptr || d_q == nullptr || d_ws == nullptr || n == 0 ||
+      ((reinterpret_cast<uintptr_t>(d_x) | reinterpret_cast<uintptr_t>(d_y)) & 3u) ||
+      (reinterpret_cast<uintptr_t>(d_q) & 7u) || (reinterpret_cast<uintptr_t>(d_ws) & 15u) || bound != bound)
+    return CUSZP_EINVAL;
+  if (ws_bytes < cuszp_quality_workspace_bytes()) return CUSZP_ENOSPACE;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  QualityArgs a{d_x, d_y, n, bound, reinterpret_cast<double*>(d_q), d_ws};
+  const uint64_t want = (n / 8 + 255) / 256;   // two float4 pairs per thread at most
+  uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_quality > 0 ? di.occ_quality : 1);
+  if (grid > want) grid = want;
+  if (grid > uint64_t(kQualityMaxGrid)) grid = kQualityMaxGrid;
+  if (grid < 1) grid = 1;
+  quality_kernel<<<unsigned(grid), 256, 0, static_cast<cudaStream_t>(stream)>>>(a);
   return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 

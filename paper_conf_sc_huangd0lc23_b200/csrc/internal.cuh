@@ -410,7 +410,18 @@ struct RangeArgs {
   WsCtrl* ws;
 };
 
+struct QualityArgs {
+  const float* x;            // original
+  const float* y;            // reconstruction
+  uint64_t n;
+  double bound;              // count |x - y| > bound (negative: counts every point with |x - y| > bound)
+  double* out;               // cuszp_quality on the device (14 x 8 bytes)
+  void* ws;                  // [0,128) counter, then one 128-byte partial per CTA
+};
+constexpr int kQualityMaxGrid = 2048;
+
 __global__ void compress_kernel(CompressArgs a);
+__global__ void quality_kernel(QualityArgs a);
 __global__ void decompress_kernel(DecompressArgs a);
 __global__ void range_kernel(RangeArgs a);
 size_t compress_smem_bytes();

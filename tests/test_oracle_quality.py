@@ -1,0 +1,115 @@
+"""Pins of oracle.quality against what the paper
+and the mathematics fix -- not against a retyped formula:
+
+* the artifact's printed compareData output for the NYX
+  temperature field: its PSNR, NRMSE, max relative error and normErr are
+  reproduced from inputs constructed to have the printed range and RMSE;
+* closed forms on inputs with exactly known errors (every e_i = +-d with d a
+  power of two, so MSE = d^2 exactly);
+* numpy's corrcoef (a library routine) for the Pearson coefficient;
+* brute-force counting for n_over_bound and exact max for the max errors.
+"""
+from __future__ import annotations
+
+import math
+
+import numpy as np
+
+import oracle
+
+# P:1920-1928 (artifact, NYX temperature.f32, 512^3 points)
+P_MIN, P_MAX = 2280.975830078125, 4782583.5
+P_RANGE = 4780302.524169921875
+P_MAX_ABS = 478.0390625
+P_MAX_REL = 0.000100
+P_PSNR = 84.770561
+P_NRMSE = 5.7739355526161066342e-05
+P_NORM_ERR = 3197659.788566
+P_N = 512 ** 3
+
+
+def test_printed_artifact_values_are_consistent():
+    # the printed numbers themselves satisfy the definitions the oracle uses
+    assert P_MAX - P_MIN == P_RANGE
+    assert abs(P_MAX_ABS / P_RANGE - P_MAX_REL) < 5e-7
+    assert abs(-20 * math.log10(P_NRMSE) - P_PSNR) < 5e-6
+    assert abs(P_NRMSE * P_RANGE * math.sqrt(P_N) - P_NORM_ERR) / P_NORM_ERR < 1e-9
+
+
+def test_oracle_reproduces_printed_psnr_nrmse():
+    # x carries the printed min / max (zero error there); every other point
+    # is 3000.0 reconstructed as 3000 +- d with d the printed RMSE rounded to
+    # the fp32 grid at 3000 (ulp 2^-12), so y is exact and e_i = -+d.
+    n = 1 << 16
+    d = round(P_NRMSE * P_RANGE * 4096) / 4096
+    x = np.full(n, 3000.0, np.float32)
+    x[0], x[1] = P_MIN, P_MAX
+    y = x.copy()
+    sgn = np.where(np.arange(n) % 2 == 0, 1.0, -1.0)
+    y[2:] = (x[2:].astype(np.float64) + sgn[2:] * d).astype(np.float32)
+    assert np.all(np.abs(x[2:].astype(np.float64) - y[2:].astype(np.float64)) == d)
+    q = oracle.quality(x, y)
+    mse = d * d * (n - 2) / n
+    assert q["min"] == P_MIN and q["max"] == P_MAX and q["range"] == P_RANGE
+    assert q["max_abs_err"] == d
+    assert abs(q["mse"] - mse) <= 1e-12 * mse
+    # printed PSNR / NRMSE up to the RMSE change of the construction
+    rmse_ratio = math.sqrt(mse) / (P_NRMSE * P_RANGE)
+    assert abs(q["psnr"] - (P_PSNR - 20 * math.log10(rmse_ratio))) < 2e-6
+    assert abs(q["nrmse"] / rmse_ratio - P_NRMSE) < 1e-12
+    assert abs(q["norm_err"] - d * math.sqrt(n - 2)) <= 1e-9 * q["norm_err"]
+
+
+def test_closed_forms_power_of_two_errors():
+    rng = np.random.default_rng(11)
+    n = 10_007
+    x = rng.integers(-1000, 1000, n).astype(np.float32)   # small integers: y = x +- 1/8 exact
+    e = np.where(rng.random(n) < 0.5, 0.125, -0.125)
+    e[::97] = 0.0
+    y = (x.astype(np.float64) - e).astype(np.float32)
+    q = oracle.quality(x, y, bound=0.1)
+    k = int(np.count_nonzero(e))
+    assert q["max_abs_err"] == 0.125
+    assert q["mse"] == 0.125 ** 2 * k / n
+    assert q["norm_err"] == math.sqrt(0.125 ** 2 * k)
+    rng_ = float(x.max()) - float(x.min())
+    assert q["range"] == rng_ and q["max_rel_err"] == 0.125 / rng_
+    assert abs(q["psnr"] - (20 * math.log10(rng_) - 10 * math.log10(q["mse"]))) < 1e-12
+    assert q["n_over_bound"] == k and q["n"] == n
+    nz = x != 0
+    assert q["max_pw_rel_err"] == float(np.max(np.abs(e[nz]) / np.abs(x[nz].astype(np.float64))))
+    assert abs(q["norm_err_norm"] - math.sqrt(0.125 ** 2 * k) / math.sqrt(float(np.sum(x.astype(np.float64) ** 2)))) < 1e-15
+
+
+def test_pearson_against_numpy_corrcoef():
+    rng = np.random.default_rng(12)
+    for n in (2, 3, 100, 5000):
+        x = rng.standard_normal(n).astype(np.float32) * 300 + 250   # offset field, like Hurricane TC
+        y = (x + rng.standard_normal(n).astype(np.float32)).astype(np.float32)
+        q = oracle.quality(x, y)
+        ref = np.corrcoef(x.astype(np.float64), y.astype(np.float64))[0, 1]
+        assert abs(q["pearson"] - ref) < 1e-12, (n, q["pearson"], ref)
+
+
+def test_lossless_and_degenerate():
+    x = np.linspace(-3, 5, 1000, dtype=np.float32)
+    q = oracle.quality(x, x.copy(), bound=0.0)
+    assert q["max_abs_err"] == 0 and q["mse"] == 0 and q["psnr"] == math.inf and q["n_over_bound"] == 0
+    # point-wise relative error skips x = 0
+    x = np.array([0.0, 2.0], np.float32)
+    y = np.array([1.0, 2.5], np.float32)
+    q = oracle.quality(x, y)
+    assert q["max_abs_err"] == 1.0 and q["max_pw_rel_err"] == 0.25
+
+
+def test_round_trip_bound_count_matches_bruteforce():
+    # on a real round trip the count of |e| > eb equals a brute-force count
+    x = np.sin(np.arange(20_000, dtype=np.float64) / 300).astype(np.float32) * 50
+    st, s = oracle.compress(x, 1e-3, oracle.REL)
+    assert st == oracle.OK
+    st, y = oracle.decompress(s, x.size)
+    eb = np.frombuffer(bytes(s[16:20]), np.float32)[0]
+    q = oracle.quality(x, y, bound=float(eb))
+    brute = int(np.count_nonzero(np.abs(x.astype(np.float64) - y.astype(np.float64)) > float(eb)))
+    assert q["n_over_bound"] == brute
+    assert q["max_abs_err"] <= float(eb) + float(np.spacing(np.abs(x)).max())
