@@ -91,16 +91,6 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
 // NaN/Inf give a NaN residual: both set `rare`, and the group is then redone
 // with the full correction (quantize_exact) -- the oracle's sequence in every
 // case.  The R5 guard |r0| < 2^22 is tracked as a running max of |r0|.
-__device__ __forceinline__ uint32_t quantize_fast(float x, float eb, float two_eb, float recip, float& rmax,
-                                                  bool& rare) {
-  const float t = __fmaf_rn(x, recip, kRoundMagic);
-  const float r0 = __fsub_rn(t, kRoundMagic);
-  rmax = fmaxf(rmax, fabsf(r0));                   // R5 guard (|r0| >= 2^22, Inf); NaN -> `rare`
-  const float res = __fmaf_rn(-r0, two_eb, x);     // exact residual (R2)
-  rare = !(fabsf(res) <= eb);
-  return __float_as_uint(t);
-}
-
 // Two elements at once with the packed fp32 pipe (FFMA2 / FADD2; same IEEE
 // RN semantics per element as the scalar sequence above).  Returns the two
 // biased integers; updates the running max |r0| (guard) and max |res|.
@@ -142,14 +132,6 @@ __device__ __forceinline__ uint32_t lorenzo_pack(uint32_t rb, int lane) {
   return (a << 1) | (uint32_t(l) >> 31);
 }
 
-// words of a block = bit length of max v = F + 1 (0 for a zero block)
-__device__ __forceinline__ uint32_t word_count(uint32_t v) {
-  const uint32_t m = __reduce_max_sync(kFull, v);
-  uint32_t b;
-  asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(m));   // 0xffffffff for m = 0
-  return b + 1;
-}
-
 }  // namespace
 
 __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(CompressArgs a) {
@@ -161,7 +143,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 
   // ---- eb_abs (Eq 1): ABS -> delta; REL -> lambda * (max - min) over the (min,max) pairs
   float eb = a.eb_in;
-  if (a.mode == CUSZP_REL) {
+  if (a.mode == CUSZP_REL && a.n_pairs == 0) {
+    eb = 0.0f;                                      // REL with n = 0 and no range (R11)
+  } else if (a.mode == CUSZP_REL) {
     float mn = a.minmax[0], mx = a.minmax[1];
     bool nan = isnan(mn) || isnan(mx);
     for (int p = 1; p < a.n_pairs; ++p) {
@@ -427,7 +411,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       h[6] = uint8_t(final_status);
       h[7] = 5;
       *reinterpret_cast<uint64_t*>(h + 8) = a.n;
-      *reinterpret_cast<float*>(h + 16) = a.n > 0 ? eb : (a.mode == CUSZP_REL ? 0.0f : a.eb_in);
+      // R11: n = 0 records the bound that would have been used (a sharded
+      // REL shard's global lambda * range; 0 for a lone empty REL array)
+      *reinterpret_cast<float*>(h + 16) = a.mode == CUSZP_REL ? eb : a.eb_in;
       *reinterpret_cast<float*>(h + 20) = a.eb_in;
       *reinterpret_cast<uint64_t*>(h + 24) = payload_bytes;
       if (a.out_bytes) *a.out_bytes = (a.n == 0) ? uint64_t(kHdr) : p0 + payload_bytes;

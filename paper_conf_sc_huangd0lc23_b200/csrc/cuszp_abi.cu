@@ -171,8 +171,8 @@ int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out,
       const int st = cuszp_range(d_in, n, nullptr, d_ws, ws_bytes, stream);
       if (st != CUSZP_OK) return st;
     }
-    return launch_compress(d_in, n, CUSZP_REL, eb, ws->minmax, 1, d_out, out_capacity, d_out_bytes,
-                           d_ws, ws_bytes, s);
+    return launch_compress(d_in, n, CUSZP_REL, eb, n > 0 ? ws->minmax : nullptr, n > 0 ? 1 : 0, d_out,
+                           out_capacity, d_out_bytes, d_ws, ws_bytes, s);
   }
   return CUSZP_EINVAL;
 }

@@ -13,9 +13,18 @@ exchanges (both stream-ordered, no host synchronisation):
     which the container header (per-shard n, bytes, offsets) is built.
 
 Every shard's decompressed floats equal the single-GPU result bit for bit
-(same eb_abs, block-aligned slabs).  Moving the compressed payloads into
-one concatenated buffer is SURVEY 8(f) NEXT rank 1; ``assemble_container``
-does it for a gathered set of shard streams.
+(same eb_abs, block-aligned slabs).
+
+SURVEY 8(f) NEXT rank 1 -- one concatenated stream and distributed
+decompression:
+ 3. ``gather_container``: the shard streams are moved into ONE container
+    buffer (header words + every shard at a 16-byte aligned offset) on one
+    rank (NCCL point-to-point receives straight into the slices) or on every
+    rank (one NCCL broadcast per shard into its slice);
+ 4. ``decompress_container``: decompresses all shards of a container on one
+    GPU (one launch per shard, each writing its slab of the output), and
+    ``decompress_sharded`` + ``allgather_slabs`` decompress a container
+    across P GPUs, rank p taking shard p.
 """
 from __future__ import annotations
 
@@ -27,7 +36,7 @@ import torch.distributed as dist
 
 BLOCK = 32
 CONTAINER_MAGIC = 0x544E4F43505A5343  # "CSZPCONT" little-endian
-CONTAINER_VERSION = 1
+CONTAINER_VERSION = 2        # v2: shard offsets and the payload base 16-byte aligned
 
 
 def slab_bounds(n_total: int, rank: int, world: int) -> tuple[int, int]:
@@ -69,14 +78,16 @@ def container_header(shard_n: list[int], sizes_all: torch.Tensor) -> torch.Tenso
     P = len(shard_n)
     dev = sizes_all.device
     n = torch.tensor(shard_n, dtype=torch.int64, device=dev)
-    offs = torch.cumsum(sizes_all, 0) - sizes_all
+    padded = (sizes_all.to(torch.int64) + 15) // 16 * 16    # every shard 16-byte aligned (TMA sources)
+    offs = torch.cumsum(padded, 0) - padded
     head = torch.tensor([CONTAINER_MAGIC - (1 << 64) if CONTAINER_MAGIC >= 1 << 63 else CONTAINER_MAGIC,
                          CONTAINER_VERSION, P, int(sum(shard_n))], dtype=torch.int64, device=dev)
     return torch.cat([head, n, sizes_all.to(torch.int64), offs])
 
 
 def container_header_bytes(P: int) -> int:
-    return 8 * (4 + 3 * P)
+    """Bytes before the first shard: the header words, padded to 16."""
+    return (8 * (4 + 3 * P) + 15) // 16 * 16
 
 
 @dataclass
@@ -138,7 +149,8 @@ def assemble_container(header_words, shard_streams: list[bytes]) -> bytes:
     h = parse_container_header(header_words)
     head = struct.pack(f"<{4 + 3 * h['P']}Q", *[int(v) & ((1 << 64) - 1) for v in
                                                 (header_words.tolist() if hasattr(header_words, "tolist") else header_words)])
-    body = bytearray(sum(h["bytes"]))
+    head = head + bytes(container_header_bytes(h["P"]) - len(head))
+    body = bytearray(container_total_bytes(h) - len(head))
     for p, s in enumerate(shard_streams):
         assert len(s) == h["bytes"][p]
         body[h["offsets"][p]:h["offsets"][p] + len(s)] = s
@@ -151,3 +163,140 @@ def split_container(buf: bytes) -> tuple[dict, list[bytes]]:
     h = parse_container_header(words)
     base = container_header_bytes(P)
     return h, [buf[base + o: base + o + b] for o, b in zip(h["offsets"], h["bytes"])]
+
+
+def container_total_bytes(h: dict) -> int:
+    """Length of the container described by a parsed header."""
+    if h["P"] == 0:
+        return container_header_bytes(0)
+    return container_header_bytes(h["P"]) + h["offsets"][-1] + h["bytes"][-1]
+
+
+def _header_bytes_tensor(header_words: torch.Tensor) -> torch.Tensor:
+    raw = header_words.contiguous().view(torch.uint8)
+    P = (header_words.numel() - 4) // 3
+    pad = container_header_bytes(P) - raw.numel()
+    return torch.cat([raw, torch.zeros(pad, dtype=torch.uint8, device=raw.device)]) if pad else raw
+
+
+def gather_container(res: ShardResult, group=None, dst: int | None = None) -> torch.Tensor | None:
+    """Materialise the concatenated container (header + every shard stream)
+    from the sharded compression result.
+
+    dst=None: on every rank (one broadcast per shard, straight into that
+    shard's slice of the container); dst=r: only on rank r (point-to-point
+    receives into the slices; other ranks send and return None).  One host
+    read of the P all-gathered sizes (8 B each) sizes the slices."""
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    h = parse_container_header(res.header.cpu())
+    base = container_header_bytes(world)
+    total = container_total_bytes(h)
+    dev = res.stream.device
+    mine = res.stream[: h["bytes"][rank]]
+    if dst is not None and rank != dst:
+        if h["bytes"][rank]:
+            dist.send(mine.contiguous(), dst=dist.get_global_rank(group, dst) if group is not None else dst,
+                      group=group)
+        return None
+    buf = torch.zeros(total, dtype=torch.uint8, device=dev)
+    buf[:base] = _header_bytes_tensor(res.header)
+    views = [buf[base + o: base + o + b] for o, b in zip(h["offsets"], h["bytes"])]
+    views[rank].copy_(mine)
+    if dst is None:
+        for p in range(world):
+            if h["bytes"][p]:
+                src = dist.get_global_rank(group, p) if group is not None else p
+                dist.broadcast(views[p], src=src, group=group)
+    else:
+        ops = []
+        for p in range(world):
+            if p != rank and h["bytes"][p]:
+                src = dist.get_global_rank(group, p) if group is not None else p
+                ops.append(dist.P2POp(dist.irecv, views[p], src, group))
+        if ops:
+            for w in dist.batch_isend_irecv(ops):
+                w.wait()
+    return buf
+
+
+def container_shards(buf: torch.Tensor) -> tuple[dict, list[torch.Tensor]]:
+    """Parsed header and the shard streams (views into buf) of a container
+    held in a device (or host) uint8 tensor.  Reads the header words only."""
+    P = int(buf[16:24].cpu().view(torch.int64).item())
+    words = buf[: 8 * (4 + 3 * P)].cpu().view(torch.int64)
+    h = parse_container_header(words)
+    base = container_header_bytes(P)
+    return h, [buf[base + o: base + o + b] for o, b in zip(h["offsets"], h["bytes"])]
+
+
+def _cuda_decompress(stream: torch.Tensor, n: int, out: torch.Tensor):
+    import paper_conf_sc_huangd0lc23_b200 as cz
+
+    return cz.decompress(stream, n, out=out, in_bytes=stream.numel())
+
+
+def decompress_container(buf: torch.Tensor, out: torch.Tensor | None = None, decompress_fn=None) -> torch.Tensor:
+    """Decompress every shard of a container on ONE device into the full
+    array (shard p -> its block-aligned slab of ``out``)."""
+    decompress_fn = decompress_fn or _cuda_decompress
+    h, shards = container_shards(buf)
+    if out is None:
+        out = torch.empty(h["n_total"], dtype=torch.float32, device=buf.device)
+    s0 = 0
+    for n_p, sh in zip(h["n"], shards):
+        if n_p:
+            decompress_fn(sh, n_p, out[s0: s0 + n_p])
+        s0 += n_p
+    return out
+
+
+def decompress_sharded(buf: torch.Tensor, group=None, decompress_fn=None) -> torch.Tensor:
+    """Distributed decompression: rank p decompresses shard p of the
+    container (present on every rank, e.g. from gather_container) into its
+    slab; returns the local slab."""
+    decompress_fn = decompress_fn or _cuda_decompress
+    rank = dist.get_rank(group)
+    h, shards = container_shards(buf)
+    n_p = h["n"][rank]
+    out = torch.empty(n_p, dtype=torch.float32, device=buf.device)
+    if n_p:
+        decompress_fn(shards[rank], n_p, out)
+    return out
+
+
+def allgather_slabs(local: torch.Tensor, shard_n: list[int], group=None) -> torch.Tensor:
+    """Every rank's decompressed slab -> the full array on every rank
+    (all-gather of equal, padded slabs, then the padding dropped)."""
+    world = dist.get_world_size(group)
+    m = max(shard_n) if shard_n else 0
+    padded = torch.zeros(m, dtype=local.dtype, device=local.device)
+    padded[: local.numel()] = local
+    allp = torch.empty(world * m, dtype=local.dtype, device=local.device)
+    _allgather(allp, padded, group)
+    return torch.cat([allp[p * m: p * m + shard_n[p]] for p in range(world)])
+
+
+def compress_to_container(x: torch.Tensor, rel: float, P: int) -> torch.Tensor:
+    """Single-device construction of a P-shard container of x (REL against
+    x's global range): the same bytes P ranks would produce with
+    compress_sharded + gather_container."""
+    import paper_conf_sc_huangd0lc23_b200 as cz
+
+    n = x.numel()
+    mm = cz.value_range(x)
+    streams, sizes, shard_n = [], [], []
+    for p in range(P):
+        s0, s1 = slab_bounds(n, p, P)
+        shard_n.append(s1 - s0)
+        out, nb = cz.compress_minmax(x[s0:s1], rel, mm)    # an empty slab is a 32-byte stream (R11)
+        streams.append(out)
+        sizes.append(nb.view(1).to(torch.int64))
+    hdr = container_header(shard_n, torch.cat(sizes))
+    h = parse_container_header(hdr.cpu())
+    base = container_header_bytes(P)
+    buf = torch.zeros(container_total_bytes(h), dtype=torch.uint8, device=x.device)
+    buf[:base] = _header_bytes_tensor(hdr)
+    for p in range(P):
+        buf[base + h["offsets"][p]: base + h["offsets"][p] + h["bytes"][p]] = streams[p][: h["bytes"][p]]
+    return buf

@@ -113,3 +113,61 @@ def test_slab_bounds_balanced():
             assert b[0][0] == 0 and b[-1][1] == n
             nb = [(e - s + 31) // 32 for s, e in b]
             assert max(nb) - min(nb) <= 1
+
+
+# ---- one concatenated container + distributed decompression
+
+def _oracle_decompress(stream: torch.Tensor, n: int, out: torch.Tensor):
+    st, y = oracle.decompress(stream.numpy(), n)
+    assert st == oracle.OK
+    out.copy_(torch.from_numpy(y))
+    return out
+
+
+def _worker_gather(rank, world, port, n, rel, outdir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    x = _field(n)
+    s0, s1 = czd.slab_bounds(n, rank, world)
+    shard_n = [b - a for a, b in (czd.slab_bounds(n, p, world) for p in range(world))]
+    res = czd.compress_sharded(torch.from_numpy(x[s0:s1].copy()), rel, shard_n,
+                               range_fn=_oracle_range, compress_fn=_oracle_compress)
+    buf_all = czd.gather_container(res)                 # on every rank
+    buf_root = czd.gather_container(res, dst=world - 1)  # on the last rank only
+    local = czd.decompress_sharded(buf_all, decompress_fn=_oracle_decompress)
+    full = czd.allgather_slabs(local, shard_n)
+    with open(os.path.join(outdir, f"g{rank}.pkl"), "wb") as f:
+        pickle.dump(dict(buf_all=buf_all.numpy().tobytes(),
+                         buf_root=None if buf_root is None else buf_root.numpy().tobytes(),
+                         stream=res.stream[: int(res.nbytes.item())].numpy().tobytes(),
+                         full=full.numpy().tobytes()), f)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,n", [(2, 100_000), (3, 70_001), (3, 40)])
+def test_gather_container_and_distributed_decompress_gloo(tmp_path, world, n):
+    rel = 1e-3
+    port = _free_port()
+    mp.spawn(_worker_gather, args=(world, port, n, rel, str(tmp_path)), nprocs=world, join=True)
+    rs = [pickle.load(open(tmp_path / f"g{p}.pkl", "rb")) for p in range(world)]
+    # the gathered container is identical on every rank and on the root, and
+    # holds every rank's stream at a 16-byte aligned offset
+    for r in rs:
+        assert r["buf_all"] == rs[0]["buf_all"]
+    assert rs[-1]["buf_root"] == rs[0]["buf_all"]
+    assert all(r["buf_root"] is None for r in rs[:-1])
+    h, shards = czd.split_container(rs[0]["buf_all"])
+    assert [bytes(s) for s in shards] == [r["stream"] for r in rs]
+    assert all(o % 16 == 0 for o in h["offsets"]) and czd.container_header_bytes(world) % 16 == 0
+    # distributed decompression + slab all-gather == whole-array REL result, bit for bit
+    x = _field(n)
+    st, whole = oracle.compress(x, rel, oracle.REL)
+    st, y_whole = oracle.decompress(whole, n)
+    for r in rs:
+        assert np.array_equal(np.frombuffer(r["full"], np.uint32), y_whole.view(np.uint32))
+    # single-device decompression of the whole container agrees too
+    y1 = czd.decompress_container(torch.frombuffer(bytearray(rs[0]["buf_all"]), dtype=torch.uint8),
+                                  decompress_fn=_oracle_decompress)
+    assert np.array_equal(y1.numpy().view(np.uint32), y_whole.view(np.uint32))
