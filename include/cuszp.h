@@ -137,6 +137,29 @@ int cuszp_decompress_host(const void* h_in, size_t in_bytes, float* h_out, size_
                           void* d_in_scratch, float* d_out_scratch,
                           void* d_ws, size_t ws_bytes, void* stream);
 
+/* Fully ASYNCHRONOUS host-buffer calls (stream-ordered, no host sync), so
+ * consecutive calls on different streams overlap both directions of the
+ * host link.  h_in of compress and h_out of decompress: pinned host memory
+ * (bulk copies on the copy engines).  h_out / h_out_bytes of compress and
+ * h_in of decompress: pinned AND device-mapped host memory (cudaHostAlloc;
+ * any pinned allocation under unified addressing): the compressed stream,
+ * whose length only the device knows, is moved by an SM copy kernel that
+ * reads that length on the device -- exactly the stream's bytes cross the
+ * link.  compress: out_capacity >= cuszp_max_compressed_bytes(n) (else
+ * ENOSPACE); *h_out_bytes receives the stream length when the stream
+ * completes.  decompress: the stream's length is taken from its own header
+ * (at most in_capacity bytes are read; d_in_scratch holds in_capacity).
+ * Sync errors: EINVAL (NULL or unmapped buffers), ENOSPACE, ECUDA; data
+ * errors are asynchronous as for the device calls.  One workspace per
+ * stream. */
+int cuszp_compress_host_async(const float* h_in, size_t n, float eb, int mode,
+                              void* h_out, size_t out_capacity, unsigned long long* h_out_bytes,
+                              float* d_in_scratch, void* d_out_scratch,
+                              void* d_ws, size_t ws_bytes, void* stream);
+int cuszp_decompress_host_async(const void* h_in, size_t in_capacity, float* h_out, size_t n,
+                                void* d_in_scratch, float* d_out_scratch,
+                                void* d_ws, size_t ws_bytes, void* stream);
+
 /* ---- reconstruction quality on the device ----
  * The statistics the paper's artifact reads off QCAT compareData
  * (P:1918-1933), PSNR as in sec 2.1, all in fp64.  x = original,

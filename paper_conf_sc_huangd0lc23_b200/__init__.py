@@ -29,6 +29,7 @@ __all__ = [
     "ABS", "REL", "Workspace", "compress", "compress_minmax", "decompress", "value_range",
     "max_compressed_bytes", "workspace_bytes", "last_status", "read_header", "compress_host",
     "decompress_host", "CuszpError", "exact_bytes_from_F", "quality", "QUALITY_KEYS",
+    "compress_host_async", "decompress_host_async",
 ]
 
 
@@ -238,3 +239,30 @@ def quality(x: torch.Tensor, y: torch.Tensor, bound: float = -1.0, out: torch.Te
     cnt = raw[12:].view(torch.int64)
     d["n"], d["n_over_bound"] = int(cnt[0]), int(cnt[1])
     return d
+
+
+def _hptr(t) -> int:
+    return t.data_ptr() if isinstance(t, torch.Tensor) else t.ctypes.data
+
+
+def compress_host_async(h_in: torch.Tensor, eb: float, mode, h_out: torch.Tensor, h_len: torch.Tensor,
+                        d_in_scratch: torch.Tensor, d_out_scratch: torch.Tensor, ws: Workspace, stream=None) -> None:
+    """Asynchronous end-to-end compression (cuszp_compress_host_async):
+    pinned h_in -> device -> stream into the pinned, mapped h_out; its length
+    into h_len (pinned int64[1]) once ``stream`` reaches this point."""
+    n_out = h_out.numel() if isinstance(h_out, torch.Tensor) else h_out.size
+    check(lib().cuszp_compress_host_async(_hptr(h_in), h_in.numel(), float(eb), _mode(mode), _hptr(h_out),
+                                          n_out, _hptr(h_len), d_in_scratch.data_ptr(),
+                                          d_out_scratch.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
+          "cuszp_compress_host_async")
+
+
+def decompress_host_async(h_in: torch.Tensor, h_out: torch.Tensor, d_in_scratch: torch.Tensor,
+                          d_out_scratch: torch.Tensor, ws: Workspace, stream=None, in_capacity: int | None = None) -> None:
+    """Asynchronous end-to-end decompression (cuszp_decompress_host_async)
+    of the stream in the pinned, mapped h_in (length from its header) into
+    the pinned h_out (n = h_out.numel())."""
+    cap = min(h_in.numel(), d_in_scratch.numel()) if in_capacity is None else int(in_capacity)
+    check(lib().cuszp_decompress_host_async(_hptr(h_in), cap, _hptr(h_out), h_out.numel(), d_in_scratch.data_ptr(),
+                                            d_out_scratch.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
+          "cuszp_decompress_host_async")

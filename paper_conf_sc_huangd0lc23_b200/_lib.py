@@ -23,6 +23,7 @@ SYMBOLS = (
     "cuszp_range", "cuszp_compress", "cuszp_compress_minmax", "cuszp_decompress",
     "cuszp_last_status", "cuszp_read_header", "cuszp_compress_host", "cuszp_decompress_host",
     "cuszp_status_string", "cuszp_version", "cuszp_quality_workspace_bytes", "cuszp_quality",
+    "cuszp_compress_host_async", "cuszp_decompress_host_async",
 )
 
 _lock = threading.Lock()
@@ -65,6 +66,10 @@ def _declare(h):
     h.cuszp_quality_workspace_bytes.restype = sz
     h.cuszp_quality.argtypes = [vp, vp, sz, C.c_double, vp, vp, sz, vp]
     h.cuszp_quality.restype = i32
+    h.cuszp_compress_host_async.argtypes = [vp, sz, f32, i32, vp, sz, vp, vp, vp, vp, sz, vp]
+    h.cuszp_compress_host_async.restype = i32
+    h.cuszp_decompress_host_async.argtypes = [vp, sz, vp, sz, vp, vp, vp, sz, vp]
+    h.cuszp_decompress_host_async.restype = i32
     h.cuszp_version.argtypes = []
     h.cuszp_version.restype = i32
 

@@ -282,6 +282,61 @@ int cuszp_decompress_host(const void* h_in, size_t in_bytes, float* h_out, size_
   return CUSZP_OK;
 }
 
+namespace {
+// device-visible address of a host-mapped pinned buffer (nullptr if not mapped)
+void* mapped(const void* h) {
+  void* d = nullptr;
+  if (h == nullptr || cudaHostGetDevicePointer(&d, const_cast<void*>(h), 0) != cudaSuccess) {
+    cudaGetLastError();   // clear the sticky-free error state of the failed query
+    return nullptr;
+  }
+  return d;
+}
+}  // namespace
+
+int cuszp_compress_host_async(const float* h_in, size_t n, float eb, int mode, void* h_out, size_t out_capacity,
+                              unsigned long long* h_out_bytes, float* d_in_scratch, void* d_out_scratch, void* d_ws,
+                              size_t ws_bytes, void* stream) {
+  if ((n > 0 && (h_in == nullptr || d_in_scratch == nullptr)) || d_out_scratch == nullptr || d_ws == nullptr)
+    return CUSZP_EINVAL;
+  if (out_capacity < cuszp_max_compressed_bytes(n)) return CUSZP_ENOSPACE;
+  void* out_dev = mapped(h_out);
+  unsigned long long* len_dev = static_cast<unsigned long long*>(mapped(h_out_bytes));
+  if (out_dev == nullptr || len_dev == nullptr) return CUSZP_EINVAL;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (n > 0 && cudaMemcpyAsync(d_in_scratch, h_in, n * sizeof(float), cudaMemcpyHostToDevice, s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  unsigned long long* d_len = reinterpret_cast<unsigned long long*>(&static_cast<WsCtrl*>(d_ws)->pad[2]);
+  int st = cuszp_compress(d_in_scratch, n, eb, mode, d_out_scratch, cuszp_max_compressed_bytes(n), d_len, d_ws,
+                          ws_bytes, stream);
+  if (st != CUSZP_OK) return st;
+  // exactly the stream's bytes cross the link; its length lands in *h_out_bytes
+  return launch_copy_len(out_dev, d_out_scratch, d_len, out_capacity, len_dev, di.sms, s);
+}
+
+int cuszp_decompress_host_async(const void* h_in, size_t in_capacity, float* h_out, size_t n, void* d_in_scratch,
+                                float* d_out_scratch, void* d_ws, size_t ws_bytes, void* stream) {
+  if (h_in == nullptr || d_in_scratch == nullptr || d_ws == nullptr ||
+      (n > 0 && (h_out == nullptr || d_out_scratch == nullptr)))
+    return CUSZP_EINVAL;
+  if (in_capacity < size_t(kHdr)) return CUSZP_EINVAL;
+  const void* in_dev = mapped(h_in);
+  if (in_dev == nullptr) return CUSZP_EINVAL;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  unsigned long long* d_len = reinterpret_cast<unsigned long long*>(&static_cast<WsCtrl*>(d_ws)->pad[4]);
+  int st = launch_stream_len(in_dev, n, d_len, s);                        // length from the stream's header
+  if (st == CUSZP_OK) st = launch_copy_len(d_in_scratch, in_dev, d_len, in_capacity, nullptr, di.sms, s);
+  if (st == CUSZP_OK) st = cuszp_decompress(d_in_scratch, in_capacity, d_out_scratch, n, d_ws, ws_bytes, stream);
+  if (st != CUSZP_OK) return st;
+  if (n > 0 && cudaMemcpyAsync(h_out, d_out_scratch, n * sizeof(float), cudaMemcpyDeviceToHost, s) != cudaSuccess)
+    return CUSZP_ECUDA;
+  return CUSZP_OK;
+}
+
 const char* cuszp_status_string(int status) {
   switch (status) {
     case CUSZP_OK: return "CUSZP_OK";
