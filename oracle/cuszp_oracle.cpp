@@ -322,7 +322,7 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
 }
 
 /* Reconstruction quality, each statistic written out by its definition
- * (DESIGN.md sec 10): the printed artifact values of P:1918-1933 satisfy
+ * (DESIGN.md sec 9.2): the printed artifact values of P:1918-1933 satisfy
  * exactly these relations (tests/test_oracle_quality.py pins them). */
 void oracle_quality(const float* x, const float* y, uint64_t n, double bound, double out[12],
                     uint64_t out_counts[2]) {

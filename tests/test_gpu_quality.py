@@ -7,7 +7,7 @@ or count of identically rounded fp64 values).  Sums are folded in another
 order (per-thread, shifted by x[0], then a fixed tree): the fp64 sums of n
 terms differ by at most ~n * 2^-53 relative to the sum of magnitudes, so
 mse, psnr, nrmse, norm_err and norm_err_norm are compared with rtol 1e-9 and
-the Pearson coefficient with atol 1e-9 (DESIGN.md sec 10)."""
+the Pearson coefficient with atol 1e-9 (DESIGN.md sec 9.2)."""
 from __future__ import annotations
 
 import math
