@@ -44,6 +44,9 @@ namespace {
 #ifndef CUSZP_C_POLL_NS
 #define CUSZP_C_POLL_NS 32
 #endif
+#ifndef CUSZP_C_LB_DELAY
+#define CUSZP_C_LB_DELAY 1500   // ns before a writer's first look-back poll (tile still loading/encoding)
+#endif
 #ifndef CUSZP_C_MINBLOCKS
 #define CUSZP_C_MINBLOCKS 3
 #endif
@@ -209,6 +212,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           if (tma_bytes) tma_load_1d(sm.in[s], a.in + e0, tma_bytes, &sm.full[s]);
         }
       }
+
     } else if (warp < kFirstCompute) {
       // --------------------------------------- writers (CTA-local tiles j = k, k+W, ...)
       for (uint32_t j = uint32_t(warp - 1);; j += kWriters) {
@@ -221,6 +225,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const uint32_t t = sm.tix[j % kTix];
         if (t == kSentinel) break;
         uint32_t nw = 0, ns = 0;
+#if CUSZP_C_LB_DELAY > 0
+        // the tile itself needs a load and an encode (> 4 us) before its
+        // prefix matters: do not poll predecessors that early
+        __nanosleep(CUSZP_C_LB_DELAY);
+#endif
         const uint64_t t_lb = a.trace ? global_ns() : 0;
         const uint64_t excl = resolve_excl(a.status, t, epoch, &nw, &ns);
         mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
@@ -270,11 +279,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
-#ifdef CUSZP_C_POLL
-        while (!mbar_test(&sm.full[s], (i / kStages) & 1u)) __nanosleep(CUSZP_C_POLL_NS);
-#else
         mbar_wait(&sm.full[s], (i / kStages) & 1u);         // suspending wait: no issue slots taken
-#endif
         const uint32_t t = sm.in_tile[s];
         if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 7, global_ns());
         // meta slot m free (tile i - kMeta released)
