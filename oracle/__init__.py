@@ -71,6 +71,16 @@ def lib():
             h.oracle_decompress.argtypes = [vp, u64, vp, u64]
             h.oracle_decompress.restype = i32
             h.oracle_quality.argtypes = [vp, vp, u64, C.c_double, vp, vp]
+            h.oracle_block_lorenzo_L.argtypes = [vp, C.c_size_t, i32, vp]
+            h.oracle_encode_block_L.argtypes = [vp, i32, vp]
+            h.oracle_encode_block_L.restype = i32
+            h.oracle_decode_block_L.argtypes = [vp, i32, i32, vp]
+            h.oracle_max_compressed_bytes_L.argtypes = [u64, i32]
+            h.oracle_max_compressed_bytes_L.restype = u64
+            h.oracle_compress_L.argtypes = [vp, u64, f32, i32, i32, vp, u64, vp]
+            h.oracle_compress_L.restype = i32
+            h.oracle_compress_minmax_L.argtypes = [vp, u64, f32, vp, i32, i32, vp, u64, vp]
+            h.oracle_compress_minmax_L.restype = i32
             _lib = h
     return _lib
 
@@ -167,6 +177,56 @@ def decompress(stream, n: int) -> tuple[int, np.ndarray]:
     out = np.zeros(int(n), np.float32)
     st = lib().oracle_decompress(_ptr(s), s.size, _ptr(out), int(n))
     return st, out
+
+
+# ---- block-length variants: L in {8, 16, 32, 64, 128}
+
+def block_lorenzo_L(q, Lb: int) -> np.ndarray:
+    q = np.ascontiguousarray(q, dtype=np.int32)
+    assert q.size % Lb == 0
+    out = np.zeros_like(q)
+    lib().oracle_block_lorenzo_L(_ptr(q), q.size // Lb, int(Lb), _ptr(out))
+    return out
+
+
+def encode_block_L(l, Lb: int) -> tuple[int, bytes]:
+    l = np.ascontiguousarray(l, dtype=np.int32)
+    assert l.size == Lb
+    buf = np.zeros(25 * 16, np.uint8)
+    F = lib().oracle_encode_block_L(_ptr(l), int(Lb), _ptr(buf))
+    return F, bytes(buf[: block_bytes(F, Lb)])
+
+
+def decode_block_L(payload: bytes, F: int, Lb: int) -> np.ndarray:
+    buf = np.zeros(25 * 16, np.uint8)
+    buf[: len(payload)] = np.frombuffer(payload, np.uint8)
+    out = np.zeros(Lb, np.int32)
+    lib().oracle_decode_block_L(_ptr(buf), int(F), int(Lb), _ptr(out))
+    return out
+
+
+def max_compressed_bytes_L(n: int, Lb: int) -> int:
+    return int(lib().oracle_max_compressed_bytes_L(int(n), int(Lb)))
+
+
+def compress_L(x, eb: float, mode: int, Lb: int) -> tuple[int, np.ndarray]:
+    x = _f32(x).ravel()
+    cap = max_compressed_bytes_L(x.size, Lb)
+    out = np.zeros(cap, np.uint8)
+    nbytes = np.zeros(1, np.uint64)
+    st = lib().oracle_compress_L(_ptr(x), x.size, np.float32(eb), int(mode), int(Lb), _ptr(out), cap, _ptr(nbytes))
+    return st, out[: int(nbytes[0])].copy() if st in (OK, ERANGE) else out[:0]
+
+
+def compress_minmax_L(x, lam: float, minmax, Lb: int) -> tuple[int, np.ndarray]:
+    x = _f32(x).ravel()
+    mm = _f32(minmax).ravel()
+    cap = max_compressed_bytes_L(x.size, Lb)
+    out = np.zeros(cap, np.uint8)
+    nbytes = np.zeros(1, np.uint64)
+    st = lib().oracle_compress_minmax_L(_ptr(x), x.size, np.float32(lam), _ptr(mm), mm.size // 2, int(Lb), _ptr(out),
+                                        cap, _ptr(nbytes))
+    return st, out[: int(nbytes[0])].copy() if st in (OK, ERANGE) else out[:0]
 
 
 QUALITY_KEYS = ("min", "max", "range", "max_abs_err", "max_rel_err", "max_pw_rel_err", "mse", "psnr", "nrmse",

@@ -22,7 +22,11 @@
 
 namespace {
 
-const int L = 32;                     /* block length, R1 */
+const int L = 32;                     /* default block length, R1 */
+const int MAX_L = 128;                /* block lengths 8..128 */
+
+bool valid_block_len(int Lb) { return Lb == 8 || Lb == 16 || Lb == 32 || Lb == 64 || Lb == 128; }
+int log2_of(int Lb) { int k = 0; while ((1 << k) < Lb) ++k; return k; }
 const int HEADER_BYTES = 32;          /* R10 */
 const float GUARD = 4194304.0f;       /* 2^22, R5 */
 const int MAX_F = 24;                 /* consequence of the guard, R5 */
@@ -48,9 +52,9 @@ bool eb_usable(float eb) {
  *  0 'CSZP' | 4 version=1 | 5 mode | 6 status | 7 log2(L)=5 | 8 u64 n |
  * 16 f32 eb_abs | 20 f32 eb_in | 24 u64 payload_bytes                    */
 void write_header(uint8_t* out, uint64_t n, int mode, int status, float eb_abs,
-                  float eb_in, uint64_t payload_bytes) {
+                  float eb_in, uint64_t payload_bytes, int Lb) {
   out[0] = 'C'; out[1] = 'S'; out[2] = 'Z'; out[3] = 'P';
-  out[4] = 1; out[5] = uint8_t(mode); out[6] = uint8_t(status); out[7] = 5;
+  out[4] = 1; out[5] = uint8_t(mode); out[6] = uint8_t(status); out[7] = uint8_t(log2_of(Lb));
   put_u64(out + 8, n);
   put_f32(out + 16, eb_abs);
   put_f32(out + 20, eb_in);
@@ -61,18 +65,18 @@ void write_header(uint8_t* out, uint64_t n, int mode, int status, float eb_abs,
  * Fig 2): Quantisation and Prediction -> Fixed-length Encoding ->
  * Global Synchronization -> Block Bit-shuffle. */
 int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int mode,
-                     uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+                     uint8_t* out, uint64_t cap, uint64_t* out_bytes, int L) {
   const uint64_t nb = (n + L - 1) / L;                  /* number of blocks N */
-  if (cap < oracle_max_compressed_bytes(n)) return ORACLE_ENOSPACE;
+  if (cap < oracle_max_compressed_bytes_L(n, L)) return ORACLE_ENOSPACE;
   std::memset(out, 0, size_t(HEADER_BYTES + align16(nb)));
 
   if (n == 0) {                                         /* R11 */
-    write_header(out, 0, mode, ORACLE_OK, eb_abs, eb_in, 0);
+    write_header(out, 0, mode, ORACLE_OK, eb_abs, eb_in, 0, L);
     *out_bytes = HEADER_BYTES;
     return ORACLE_OK;
   }
   if (!eb_usable(eb_abs)) {                             /* R5 */
-    write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0);
+    write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0, L);
     *out_bytes = HEADER_BYTES + align16(nb);
     return ORACLE_ERANGE;
   }
@@ -80,14 +84,14 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
   /* (1) Pre-quantisation, the only lossy step. */
   std::vector<int32_t> r(static_cast<size_t>(nb * L), 0);            /* zero pad, R8 */
   if (oracle_prequantize(x, size_t(n), eb_abs, r.data()) != ORACLE_OK) {
-    write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0);
+    write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0, L);
     *out_bytes = HEADER_BYTES + align16(nb);
     return ORACLE_ERANGE;
   }
 
   /* (1') Lorenzo prediction inside each block. */
   std::vector<int32_t> l(static_cast<size_t>(nb * L));
-  oracle_block_lorenzo(r.data(), size_t(nb), l.data());
+  oracle_block_lorenzo_L(r.data(), size_t(nb), L, l.data());
 
   /* (2) Fixed-length encoding: F_k and CmpL_k per block,
    *     giving the BlockOffsetArray. */
@@ -95,8 +99,8 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
   std::vector<uint64_t> block_offset(static_cast<size_t>(nb));
   uint8_t* fixed_length = out + HEADER_BYTES;          /* Fig 12 part 1 */
   for (uint64_t k = 0; k < nb; ++k) {
-    uint8_t buf[4 * (MAX_F + 1)];
-    int F = oracle_encode_block(&l[size_t(k * L)], buf);
+    uint8_t buf[(MAX_L / 8) * (MAX_F + 1)];
+    int F = oracle_encode_block_L(&l[size_t(k * L)], L, buf);
     fixed_length[k] = uint8_t(F);
     block_offset[k] = oracle_block_bytes(F, L);
     encoded[k].assign(buf, buf + block_offset[k]);
@@ -114,7 +118,7 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
     if (block_offset[k] > 0)
       std::memcpy(out + p0 + sync_offset[k], encoded[k].data(), size_t(block_offset[k]));
 
-  write_header(out, n, mode, ORACLE_OK, eb_abs, eb_in, payload_bytes);
+  write_header(out, n, mode, ORACLE_OK, eb_abs, eb_in, payload_bytes, L);
   *out_bytes = p0 + payload_bytes;
   return ORACLE_OK;
 }
@@ -164,6 +168,10 @@ int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q) {
 }
 
 void oracle_block_lorenzo(const int32_t* q, size_t nb, int32_t* l) {
+  oracle_block_lorenzo_L(q, nb, L, l);
+}
+
+void oracle_block_lorenzo_L(const int32_t* q, size_t nb, int L, int32_t* l) {
   /* l_i = r_i - r_{i-1}, r_{i-1} = 0 for the first integer of each block
    * (P:525-529): the linear recurrence never crosses a block. */
   for (size_t k = 0; k < nb; ++k) {
@@ -197,11 +205,13 @@ void oracle_exclusive_scan(const uint64_t* cmpl, size_t k, uint64_t* sync_off) {
   for (size_t i = 0; i < k; ++i) { sync_off[i] = s; s += cmpl[i]; }
 }
 
-int oracle_encode_block(const int32_t l[32], uint8_t* out) {
+int oracle_encode_block(const int32_t l[32], uint8_t* out) { return oracle_encode_block_L(l, L, out); }
+
+int oracle_encode_block_L(const int32_t* l, int L, uint8_t* out) {
   /* Sign map: bit 0 for positive, 1 otherwise; integer 0 -> bit 0 (R7).
-   * L/8 = 4 bytes; element j -> byte j/8, bit j%8 (R9). */
-  uint8_t sign_map[L / 8] = {0, 0, 0, 0};
-  uint32_t mag[L];
+   * L/8 bytes; element j -> byte j/8, bit j%8 (R9). */
+  uint8_t sign_map[MAX_L / 8] = {0};
+  uint32_t mag[MAX_L];
   uint32_t max_abs = 0;
   for (int j = 0; j < L; ++j) {
     if (l[j] < 0) sign_map[j / 8] |= uint8_t(1u << (j % 8));
@@ -224,6 +234,10 @@ int oracle_encode_block(const int32_t l[32], uint8_t* out) {
 }
 
 void oracle_decode_block(const uint8_t* payload, int F, int32_t l[32]) {
+  oracle_decode_block_L(payload, F, L, l);
+}
+
+void oracle_decode_block_L(const uint8_t* payload, int F, int L, int32_t* l) {
   if (F == 0) { for (int j = 0; j < L; ++j) l[j] = 0; return; }
   for (int j = 0; j < L; ++j) {
     uint32_t mag = 0;
@@ -236,26 +250,34 @@ void oracle_decode_block(const uint8_t* payload, int F, int32_t l[32]) {
   }
 }
 
-uint64_t oracle_max_compressed_bytes(uint64_t n) {
+uint64_t oracle_max_compressed_bytes(uint64_t n) { return oracle_max_compressed_bytes_L(n, L); }
+
+uint64_t oracle_max_compressed_bytes_L(uint64_t n, int L) {
   const uint64_t nb = (n + L - 1) / L;
-  return HEADER_BYTES + align16(nb) + uint64_t(4 * (MAX_F + 1)) * nb;
+  return HEADER_BYTES + align16(nb) + uint64_t(L / 8) * uint64_t(MAX_F + 1) * nb;
 }
 
 int oracle_compress(const float* x, uint64_t n, float eb, int mode,
                     uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
-  if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr) return ORACLE_EINVAL;
+  return oracle_compress_L(x, n, eb, mode, L, out, cap, out_bytes);
+}
+
+int oracle_compress_L(const float* x, uint64_t n, float eb, int mode, int L,
+                      uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr || !valid_block_len(L))
+    return ORACLE_EINVAL;
   if (mode == 0) {                                      /* ABS: eb = delta */
     if (!eb_usable(eb)) return ORACLE_EINVAL;
-    return compress_with_eb(x, n, eb, eb, 0, out, cap, out_bytes);
+    return compress_with_eb(x, n, eb, eb, 0, out, cap, out_bytes, L);
   }
   if (mode == 1) {                                      /* REL: eb = lambda * r */
     if (!(eb > 0.0f) || !std::isfinite(eb)) return ORACLE_EINVAL;
-    if (n == 0) return compress_with_eb(x, 0, 0.0f, eb, 1, out, cap, out_bytes);
+    if (n == 0) return compress_with_eb(x, 0, 0.0f, eb, 1, out, cap, out_bytes, L);
     float mn, mx;
     oracle_value_range(x, size_t(n), &mn, &mx);
     const float range = mx - mn;                        /* R3: fp32 */
     const float eb_abs = eb * range;
-    return compress_with_eb(x, n, eb_abs, eb, 1, out, cap, out_bytes);
+    return compress_with_eb(x, n, eb_abs, eb, 1, out, cap, out_bytes, L);
   }
   return ORACLE_EINVAL;
 }
@@ -263,8 +285,14 @@ int oracle_compress(const float* x, uint64_t n, float eb, int mode,
 int oracle_compress_minmax(const float* x, uint64_t n, float lambda,
                            const float* minmax, int n_pairs,
                            uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  return oracle_compress_minmax_L(x, n, lambda, minmax, n_pairs, L, out, cap, out_bytes);
+}
+
+int oracle_compress_minmax_L(const float* x, uint64_t n, float lambda,
+                             const float* minmax, int n_pairs, int L,
+                             uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
   if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr ||
-      minmax == nullptr || n_pairs <= 0) return ORACLE_EINVAL;
+      minmax == nullptr || n_pairs <= 0 || !valid_block_len(L)) return ORACLE_EINVAL;
   if (!(lambda > 0.0f) || !std::isfinite(lambda)) return ORACLE_EINVAL;
   float mn = minmax[0], mx = minmax[1];
   for (int p = 1; p < n_pairs; ++p) {
@@ -273,7 +301,7 @@ int oracle_compress_minmax(const float* x, uint64_t n, float lambda,
   }
   const float range = mx - mn;
   const float eb_abs = lambda * range;
-  return compress_with_eb(x, n, eb_abs, lambda, 1, out, cap, out_bytes);
+  return compress_with_eb(x, n, eb_abs, lambda, 1, out, cap, out_bytes, L);
 }
 
 int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t n) {
@@ -283,7 +311,8 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
   if (in == nullptr || (n > 0 && out == nullptr)) return ORACLE_EINVAL;
   if (in_bytes < uint64_t(HEADER_BYTES)) return ORACLE_ECORRUPT;
   if (!(in[0] == 'C' && in[1] == 'S' && in[2] == 'Z' && in[3] == 'P') ||
-      in[4] != 1 || in[7] != 5) return ORACLE_ECORRUPT;
+      in[4] != 1 || in[7] < 3 || in[7] > 7) return ORACLE_ECORRUPT;
+  const int L = 1 << in[7];                             /* block length from the header */
   if (in[6] != ORACLE_OK) return in[6] == ORACLE_ERANGE ? ORACLE_ERANGE : ORACLE_ECORRUPT;
   if (get_u64(in + 8) != n) return ORACLE_EINVAL;
   if (n == 0) return ORACLE_OK;
@@ -307,8 +336,8 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
 
   const float two_eb = eb_abs + eb_abs;
   for (uint64_t k = 0; k < nb; ++k) {
-    int32_t l[L];
-    oracle_decode_block(in + p0 + sync_offset[k], fixed_length[k], l);
+    int32_t l[MAX_L];
+    oracle_decode_block_L(in + p0 + sync_offset[k], fixed_length[k], L, l);
     /* reverse Lorenzo: r_i = r_{i-1} + l_i inside the block */
     int32_t r = 0;
     for (int i = 0; i < L; ++i) {

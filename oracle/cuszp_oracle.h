@@ -93,6 +93,22 @@ int oracle_compress_minmax(const float* x, uint64_t n, float lambda,
 int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out,
                       uint64_t n);
 
+/* ---- block-length variants ---------------------
+ * The same method with block length L in {8, 16, 32, 64, 128} (the lengths
+ * of the paper's smoothness analysis; Eq 2 is CmpL = (F+1) L/8
+ * bytes, the bit-shuffle puts bit k of every |l_j| into the k-th group of
+ * L/8 bytes).  Header byte 7 = log2(L); oracle_decompress reads
+ * it.  The functions without _L are the L = 32 ones. */
+void oracle_block_lorenzo_L(const int32_t* q, size_t nb, int L, int32_t* l);
+int oracle_encode_block_L(const int32_t* l, int L, uint8_t* out);
+void oracle_decode_block_L(const uint8_t* payload, int F, int L, int32_t* l);
+uint64_t oracle_max_compressed_bytes_L(uint64_t n, int L);
+int oracle_compress_L(const float* x, uint64_t n, float eb, int mode, int L,
+                      uint8_t* out, uint64_t cap, uint64_t* out_bytes);
+int oracle_compress_minmax_L(const float* x, uint64_t n, float lambda,
+                             const float* minmax, int n_pairs, int L,
+                             uint8_t* out, uint64_t cap, uint64_t* out_bytes);
+
 /* ---- reconstruction quality -------------------
  * The statistics of the paper's artifact output (QCAT compareData,
  * P:1918-1933) and PSNR (sec 2.1), in fp64, two plain passes
