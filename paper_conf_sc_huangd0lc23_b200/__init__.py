@@ -53,8 +53,8 @@ def _require_cuda(t: torch.Tensor, name: str, dtype=None):
         raise ValueError(f"{name} must be contiguous")
 
 
-def max_compressed_bytes(n: int) -> int:
-    return int(lib().cuszp_max_compressed_bytes(int(n)))
+def max_compressed_bytes(n: int, block_len: int = BLOCK_LEN) -> int:
+    return int(lib().cuszp_max_compressed_bytes_L(int(n), int(block_len)))
 
 
 def workspace_bytes(n: int) -> int:
@@ -113,43 +113,46 @@ def value_range(x: torch.Tensor, ws: Workspace | None = None, out: torch.Tensor 
 
 
 def compress(x: torch.Tensor, eb: float, mode="rel", out: torch.Tensor | None = None,
-             out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None):
+             out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None,
+             block_len: int = BLOCK_LEN):
     """Compress a float32 CUDA tensor.  Returns (stream buffer uint8 tensor of
     capacity max_compressed_bytes(n), device int64 tensor [1] holding the
     exact stream length).  Asynchronous; data errors land in the header."""
     _require_cuda(x, "x", torch.float32)
     n = x.numel()
-    cap = max_compressed_bytes(n)
+    cap = max_compressed_bytes(n, block_len)
     if out is None:
         out = torch.empty(cap, dtype=torch.uint8, device=x.device)
     _require_cuda(out, "out", torch.uint8)
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
     ws = _workspace(n, x.device, ws)
-    check(lib().cuszp_compress(x.data_ptr(), n, float(eb), _mode(mode), out.data_ptr(), out.numel(),
-                               out_bytes.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_compress")
+    check(lib().cuszp_compress_L(x.data_ptr(), n, float(eb), _mode(mode), int(block_len), out.data_ptr(),
+                                 out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
+          "cuszp_compress")
     return out, out_bytes
 
 
 def compress_minmax(x: torch.Tensor, lam: float, minmax: torch.Tensor, out: torch.Tensor | None = None,
-                    out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None):
+                    out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None,
+                    block_len: int = BLOCK_LEN):
     """REL compression against a global range given as (min, max) pairs on the device."""
     _require_cuda(x, "x", torch.float32)
     _require_cuda(minmax, "minmax", torch.float32)
     n = x.numel()
     if out is None:
-        out = torch.empty(max_compressed_bytes(n), dtype=torch.uint8, device=x.device)
+        out = torch.empty(max_compressed_bytes(n, block_len), dtype=torch.uint8, device=x.device)
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
     ws = _workspace(n, x.device, ws)
-    check(lib().cuszp_compress_minmax(x.data_ptr(), n, float(lam), minmax.data_ptr(), minmax.numel() // 2,
-                                      out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
-                                      _stream_ptr(stream)), "cuszp_compress_minmax")
+    check(lib().cuszp_compress_minmax_L(x.data_ptr(), n, float(lam), minmax.data_ptr(), minmax.numel() // 2,
+                                        int(block_len), out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(),
+                                        ws.nbytes, _stream_ptr(stream)), "cuszp_compress_minmax")
     return out, out_bytes
 
 
 def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None, in_bytes: int | None = None,
-               ws: Workspace | None = None, stream=None) -> torch.Tensor:
+               ws: Workspace | None = None, stream=None, block_len: int = BLOCK_LEN) -> torch.Tensor:
     """Decompress a device stream into n float32 values (asynchronous)."""
     _require_cuda(stream_buf, "stream_buf", torch.uint8)
     if out is None:
@@ -157,8 +160,8 @@ def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None
     _require_cuda(out, "out", torch.float32)
     ws = _workspace(n, stream_buf.device, ws)
     nbytes = stream_buf.numel() if in_bytes is None else int(in_bytes)
-    check(lib().cuszp_decompress(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), ws.ptr(), ws.nbytes,
-                                 _stream_ptr(stream)), "cuszp_decompress")
+    check(lib().cuszp_decompress_L(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), int(block_len), ws.ptr(),
+                                   ws.nbytes, _stream_ptr(stream)), "cuszp_decompress")
     return out
 
 

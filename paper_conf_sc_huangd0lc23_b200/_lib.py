@@ -24,6 +24,7 @@ SYMBOLS = (
     "cuszp_last_status", "cuszp_read_header", "cuszp_compress_host", "cuszp_decompress_host",
     "cuszp_status_string", "cuszp_version", "cuszp_quality_workspace_bytes", "cuszp_quality",
     "cuszp_compress_host_async", "cuszp_decompress_host_async",
+    "cuszp_compress_L", "cuszp_compress_minmax_L", "cuszp_decompress_L", "cuszp_max_compressed_bytes_L",
 )
 
 _lock = threading.Lock()
@@ -70,6 +71,14 @@ def _declare(h):
     h.cuszp_compress_host_async.restype = i32
     h.cuszp_decompress_host_async.argtypes = [vp, sz, vp, sz, vp, vp, vp, sz, vp]
     h.cuszp_decompress_host_async.restype = i32
+    h.cuszp_max_compressed_bytes_L.argtypes = [sz, i32]
+    h.cuszp_max_compressed_bytes_L.restype = sz
+    h.cuszp_compress_L.argtypes = [vp, sz, f32, i32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_compress_L.restype = i32
+    h.cuszp_compress_minmax_L.argtypes = [vp, sz, f32, vp, i32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_compress_minmax_L.restype = i32
+    h.cuszp_decompress_L.argtypes = [vp, sz, vp, sz, i32, vp, sz, vp]
+    h.cuszp_decompress_L.restype = i32
     h.cuszp_version.argtypes = []
     h.cuszp_version.restype = i32
 

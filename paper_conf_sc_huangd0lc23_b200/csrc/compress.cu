@@ -134,10 +134,25 @@ __device__ __forceinline__ uint32_t lorenzo_pack(uint32_t rb, int lane) {
   const uint32_t a = uint32_t(l < 0 ? -l : l);
   return (a << 1) | (uint32_t(l) >> 31);
 }
+// same, lane 0 taking `first` (biased) as its predecessor: the last element
+// of the previous 32-element sub-block of an L = 32 M block
+__device__ __forceinline__ uint32_t lorenzo_pack_first(uint32_t rb, int lane, uint32_t first) {
+  uint32_t prev = __shfl_up_sync(kFull, rb, 1);
+  prev = lane ? prev : first;
+  const int l = int(rb - prev);
+  const uint32_t a = uint32_t(l < 0 ? -l : l);
+  return (a << 1) | (uint32_t(l) >> 31);
+}
 
 }  // namespace
 
+// M = L / 32: an L-block is M consecutive 32-element
+// sub-blocks sharing one F; word k of sub-block i of a block sits at
+// M k + i of the block's payload (a plane is L/8 bytes, element j at byte
+// j/8, bit j%8 -- R9 generalised).  M = 1 is the paper's default L = 32.
+template <int M>
 __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(CompressArgs a) {
+  static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
   extern __shared__ __align__(128) unsigned char smem_raw[];
   CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
@@ -319,8 +334,17 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
           }
           uint32_t v[4];
+          if constexpr (M == 1) {
 #pragma unroll
-          for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
+            for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
+          } else {
+            // a block continues across its sub-blocks: lane 0 of sub-block q
+            // takes lane 31 of sub-block q-1 unless q starts a block
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              v[q] = lorenzo_pack_first(r[q], lane,
+                                        (q % M == 0) ? kRoundMagicBits : __shfl_sync(kFull, r[q > 0 ? q - 1 : 0], 31));
+          }
           // room in this warp's ring for a worst-case group (4 x 25 words)
           while (head + cursor + 4 * kMaxBlockWords - ld_volatile_u32(&sm.tail[w]) > kRing)
             __nanosleep(CUSZP_C_POLL_NS);
@@ -335,11 +359,46 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(__reduce_or_sync(kFull, v[q])));   // -1 for 0
             wq[q] = b + 1;
           }
+          // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
+          // record it, and clamp so an ERANGE stream never exceeds the
+          // capacity bound (25 words per block) nor the ring reservation
+          wmax = max(wmax, max(max(wq[0], wq[1]), max(wq[2], wq[3])));
+#pragma unroll
+          for (int q = 0; q < 4; ++q) wq[q] = min(wq[q], uint32_t(kMaxBlockWords));
+          if constexpr (M == 2) {                                        // one F per block
+            wq[0] = wq[1] = max(wq[0], wq[1]);
+            wq[2] = wq[3] = max(wq[2], wq[3]);
+          } else if constexpr (M == 4) {
+            wq[0] = wq[1] = wq[2] = wq[3] = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+          }
           const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
-          wmax = max(wmax, span);                                        // > 25: NaN/Inf data (R5)
           const uint32_t wb = wq[0] | (wq[1] << 8) | (wq[2] << 16) | (wq[3] << 24);
           const uint32_t base = head + cursor;
-          if (span <= 8) {
+          if (M > 1) {
+            // word k of sub-block q -> block payload position M k + q % M
+            const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
+            if (span <= 8) {
+              const uint32_t tw = xpose(v[0] | (v[1] << 8) | (v[2] << 16) | (v[3] << 24));
+              const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
+              const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
+              if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;
+            } else if (span <= 16) {
+              const uint32_t t01 = xpose(v[0] | (v[1] << 16));
+              const uint32_t t23 = xpose(v[2] | (v[3] << 16));
+              const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
+              if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;
+              const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
+              const uint32_t sub23 = (M == 2) ? h : 2u + h;
+              if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;
+            } else {
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                const uint32_t tq = xpose(v[q]);
+                const uint32_t pre = (q & ~(M - 1)) == 0 ? 0u : __byte_perm(pb, 0, 0x4440u + (q & ~(M - 1)));
+                if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;
+              }
+            }
+          } else if (span <= 8) {
             const uint32_t tw = xpose(v[0] | (v[1] << 8) | (v[2] << 16) | (v[3] << 24));
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
             const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
@@ -363,11 +422,23 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
           // F = words - 1 (0 for a zero block), bytewise (counts <= 32, no carries)
           fpack[g] = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
+          if constexpr (M == 2) fpack[g] = __byte_perm(fpack[g], 0, 0x4420u);   // blocks (0,1), (2,3)
+          if constexpr (M == 4) fpack[g] &= 0xffu;                             // one block
         }
-        // F bytes of the warp's 16 blocks (Fig 12 part 1): one 16-byte store
-        const uint64_t blk0 = uint64_t(t) * kTileBlocks + uint64_t(w) * kBPW;
-        if (lane == 0 && blk0 < a.nb)
-          *reinterpret_cast<uint4*>(a.out + kHdr + blk0) = make_uint4(fpack[0], fpack[1], fpack[2], fpack[3]);
+        // F bytes of the warp's 16 / M blocks (Fig 12 part 1): one store; the
+        // stores also cover the F area's zero padding up to align16(nb)
+        // (padding sub-blocks past n encode as zero blocks, F = 0)
+        const uint64_t blk0 = (uint64_t(t) * kTileBlocks + uint64_t(w) * kBPW) / M;
+        if (lane == 0 && blk0 < align16(a.nb)) {
+          if constexpr (M == 1)
+            *reinterpret_cast<uint4*>(a.out + kHdr + blk0) = make_uint4(fpack[0], fpack[1], fpack[2], fpack[3]);
+          else if constexpr (M == 2)
+            *reinterpret_cast<uint2*>(a.out + kHdr + blk0) =
+                make_uint2(fpack[0] | (fpack[1] << 16), fpack[2] | (fpack[3] << 16));
+          else
+            *reinterpret_cast<uint32_t*>(a.out + kHdr + blk0) =
+                fpack[0] | (fpack[1] << 8) | (fpack[2] << 16) | (fpack[3] << 24);
+        }
         __syncwarp();
         if (lane == 0) {
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
@@ -414,7 +485,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       h[4] = CUSZP_VERSION;
       h[5] = uint8_t(a.mode);
       h[6] = uint8_t(final_status);
-      h[7] = 5;
+      h[7] = uint8_t(5 + (M == 2 ? 1 : M == 4 ? 2 : 0));   // log2(L)
       *reinterpret_cast<uint64_t*>(h + 8) = a.n;
       // R11: n = 0 records the bound that would have been used (a sharded
       // REL shard's global lambda * range; 0 for a lone empty REL array)
@@ -426,6 +497,10 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
     finish_call(a.ws, a.status, a.status_cap, epoch, final_status);
   }
 }
+
+template __global__ void compress_kernel<1>(CompressArgs);
+template __global__ void compress_kernel<2>(CompressArgs);
+template __global__ void compress_kernel<4>(CompressArgs);
 
 size_t compress_smem_bytes() { return sizeof(CompressSmem); }
 int compress_threads() { return kCThreads; }

@@ -11,12 +11,16 @@ using namespace cuszp;
 
 namespace {
 
-uint64_t num_blocks(uint64_t n) { return (n + kL - 1) / kL; }
+uint64_t num_blocks(uint64_t n, int L = kL) { return (n + L - 1) / L; }
+// M = L / 32 for the block lengths of SURVEY 8(f) rank 3 (0: unsupported)
+int sub_blocks(int L) { return L == 32 ? 1 : L == 64 ? 2 : L == 128 ? 4 : 0; }
+int mi(int M) { return M == 1 ? 0 : M == 2 ? 1 : 2; }
 uint64_t num_tiles(uint64_t n) { return (num_blocks(n) + kTileBlocks - 1) / kTileBlocks; }
 
 struct DeviceInfo {
   int sms = 0;
   int occ_compress = 0, occ_decompress = 0, occ_range = 0, occ_quality = 0;
+  int occ_c[3] = {0, 0, 0}, occ_d[3] = {0, 0, 0};   // per M = 1, 2, 4
 };
 
 // Per-device launch geometry, computed once: persistent grids of
@@ -32,15 +36,24 @@ int device_info(DeviceInfo* out) {
     DeviceInfo d;
     const int cs = int(compress_smem_bytes()), ds = int(decompress_smem_bytes());
     if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
-        cudaFuncSetAttribute(compress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
-        cudaFuncSetAttribute(decompress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess)
+        cudaFuncSetAttribute(compress_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
+        cudaFuncSetAttribute(compress_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
+        cudaFuncSetAttribute(compress_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
+        cudaFuncSetAttribute(decompress_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess ||
+        cudaFuncSetAttribute(decompress_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess ||
+        cudaFuncSetAttribute(decompress_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess)
       return CUSZP_ECUDA;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_compress, compress_kernel, compress_threads(), cs) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_decompress, decompress_kernel, decompress_threads(), ds) !=
-            cudaSuccess ||
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_c[0], compress_kernel<1>, compress_threads(), cs) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_c[1], compress_kernel<2>, compress_threads(), cs) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_c[2], compress_kernel<4>, compress_threads(), cs) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_d[0], decompress_kernel<1>, decompress_threads(), ds) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_d[1], decompress_kernel<2>, decompress_threads(), ds) != cudaSuccess ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_d[2], decompress_kernel<4>, decompress_threads(), ds) != cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_quality, quality_kernel, 256, 0) != cudaSuccess)
       return CUSZP_ECUDA;
+    d.occ_compress = d.occ_c[0];
+    d.occ_decompress = d.occ_d[0];
     cache[dev] = d;
     have[dev] = true;
   }
@@ -65,15 +78,17 @@ uint32_t status_capacity(size_t ws_bytes) {
 
 int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const float* d_minmax,
                     int n_pairs, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
-                    void* d_ws, size_t ws_bytes, cudaStream_t stream) {
-  if (out_capacity < cuszp_max_compressed_bytes(n) || ws_bytes < cuszp_workspace_bytes(n))
+                    void* d_ws, size_t ws_bytes, cudaStream_t stream, int L = kL) {
+  const int M = sub_blocks(L);
+  if (M == 0) return CUSZP_EINVAL;
+  if (out_capacity < cuszp_max_compressed_bytes_L(n, L) || ws_bytes < cuszp_workspace_bytes(n))
     return CUSZP_ENOSPACE;
   DeviceInfo di;
   if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
   CompressArgs a;
   a.in = d_in;
   a.n = n;
-  a.nb = num_blocks(n);
+  a.nb = num_blocks(n, L);
   a.num_tiles = uint32_t(num_tiles(n));
   a.mode = mode;
   a.eb_in = eb_in;
@@ -85,10 +100,13 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
   a.trace = g_trace;
-  uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_compress > 0 ? di.occ_compress : 1);
+  const int occ = di.occ_c[mi(M)];
+  uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  compress_kernel<<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
+  if (M == 1) compress_kernel<1><<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
+  else if (M == 2) compress_kernel<2><<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
+  else compress_kernel<4><<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
   return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
@@ -96,9 +114,12 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
 
 extern "C" {
 
-size_t cuszp_max_compressed_bytes(size_t n) {
-  const uint64_t nb = num_blocks(n);
-  return size_t(kHdr + align16(nb) + uint64_t(4 * (kMaxF + 1)) * nb);
+size_t cuszp_max_compressed_bytes(size_t n) { return cuszp_max_compressed_bytes_L(n, kL); }
+
+size_t cuszp_max_compressed_bytes_L(size_t n, int block_len) {
+  if (sub_blocks(block_len) == 0) return 0;
+  const uint64_t nb = num_blocks(n, block_len);
+  return size_t(kHdr + align16(nb) + uint64_t(block_len / 8) * (kMaxF + 1) * nb);
 }
 
 size_t cuszp_compressed_bytes_from_F(const uint8_t* h_F, size_t nb) {
@@ -152,7 +173,14 @@ int cuszp_quality(const float* d_x, const float* d_y, size_t n, double bound, cu
 
 int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out, size_t out_capacity,
                    unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes, void* stream) {
-  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr) return CUSZP_EINVAL;
+  return cuszp_compress_L(d_in, n, eb, mode, kL, d_out, out_capacity, d_out_bytes, d_ws, ws_bytes, stream);
+}
+
+int cuszp_compress_L(const float* d_in, size_t n, float eb, int mode, int block_len, void* d_out,
+                     size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes,
+                     void* stream) {
+  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || sub_blocks(block_len) == 0)
+    return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
@@ -160,11 +188,11 @@ int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out,
   if (mode == CUSZP_ABS) {
     if (!eb_is_normal(eb)) return CUSZP_EINVAL;
     return launch_compress(d_in, n, CUSZP_ABS, eb, nullptr, 0, d_out, out_capacity, d_out_bytes, d_ws,
-                           ws_bytes, s);
+                           ws_bytes, s, block_len);
   }
   if (mode == CUSZP_REL) {
     if (!(eb > 0.0f) || !(eb - eb == 0.0f)) return CUSZP_EINVAL;
-    if (out_capacity < cuszp_max_compressed_bytes(n) || ws_bytes < cuszp_workspace_bytes(n))
+    if (out_capacity < cuszp_max_compressed_bytes_L(n, block_len) || ws_bytes < cuszp_workspace_bytes(n))
       return CUSZP_ENOSPACE;
     const WsCtrl* ws = static_cast<const WsCtrl*>(d_ws);
     if (n > 0) {
@@ -172,7 +200,7 @@ int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out,
       if (st != CUSZP_OK) return st;
     }
     return launch_compress(d_in, n, CUSZP_REL, eb, n > 0 ? ws->minmax : nullptr, n > 0 ? 1 : 0, d_out,
-                           out_capacity, d_out_bytes, d_ws, ws_bytes, s);
+                           out_capacity, d_out_bytes, d_ws, ws_bytes, s, block_len);
   }
   return CUSZP_EINVAL;
 }
@@ -180,20 +208,33 @@ int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out,
 int cuszp_compress_minmax(const float* d_in, size_t n, float lambda, const float* d_minmax, int n_pairs,
                           void* d_out, size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws,
                           size_t ws_bytes, void* stream) {
+  return cuszp_compress_minmax_L(d_in, n, lambda, d_minmax, n_pairs, kL, d_out, out_capacity, d_out_bytes, d_ws,
+                                 ws_bytes, stream);
+}
+
+int cuszp_compress_minmax_L(const float* d_in, size_t n, float lambda, const float* d_minmax, int n_pairs,
+                            int block_len, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
+                            void* d_ws, size_t ws_bytes, void* stream) {
   if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || d_minmax == nullptr ||
-      n_pairs <= 0)
+      n_pairs <= 0 || sub_blocks(block_len) == 0)
     return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
   if (!(lambda > 0.0f) || !(lambda - lambda == 0.0f)) return CUSZP_EINVAL;
   return launch_compress(d_in, n, CUSZP_REL, lambda, d_minmax, n_pairs, d_out, out_capacity, d_out_bytes,
-                         d_ws, ws_bytes, static_cast<cudaStream_t>(stream));
+                         d_ws, ws_bytes, static_cast<cudaStream_t>(stream), block_len);
 }
 
 int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n, void* d_ws, size_t ws_bytes,
                      void* stream) {
-  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr) return CUSZP_EINVAL;
+  return cuszp_decompress_L(d_in, in_bytes, d_out, n, kL, d_ws, ws_bytes, stream);
+}
+
+int cuszp_decompress_L(const void* d_in, size_t in_bytes, float* d_out, size_t n, int block_len, void* d_ws,
+                       size_t ws_bytes, void* stream) {
+  const int M = sub_blocks(block_len);
+  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr || M == 0) return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
@@ -205,17 +246,20 @@ int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n, 
   a.in_bytes = in_bytes;
   a.out = d_out;
   a.n = n;
-  a.nb = num_blocks(n);
+  a.nb = num_blocks(n, block_len);
   a.num_tiles = uint32_t(num_tiles(n));
   a.ws = static_cast<WsCtrl*>(d_ws);
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
   a.trace = g_trace;
-  uint64_t grid = uint64_t(di.sms) * uint64_t(di.occ_decompress > 0 ? di.occ_decompress : 1);
+  const int occ = di.occ_d[mi(M)];
+  uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  decompress_kernel<<<unsigned(grid), decompress_threads(), decompress_smem_bytes(),
-                      static_cast<cudaStream_t>(stream)>>>(a);
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (M == 1) decompress_kernel<1><<<unsigned(grid), decompress_threads(), decompress_smem_bytes(), s>>>(a);
+  else if (M == 2) decompress_kernel<2><<<unsigned(grid), decompress_threads(), decompress_smem_bytes(), s>>>(a);
+  else decompress_kernel<4><<<unsigned(grid), decompress_threads(), decompress_smem_bytes(), s>>>(a);
   return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 

@@ -70,7 +70,13 @@ static_assert(kBarFree0 + 2 <= 16, "named barriers");
 
 }  // namespace
 
+// M = L / 32: see compress.cu -- sub-block i of a block
+// finds its word k at M k + i of the block's payload, and the in-block
+// prefix sum (a11) runs over the block's M sub-blocks.
+template <int M>
 __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kernel(DecompressArgs a) {
+  static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
+  constexpr uint32_t kLog2L = 5 + (M == 2 ? 1 : M == 4 ? 2 : 0);
   extern __shared__ __align__(128) unsigned char smem_raw[];
   DecompressSmem& sm = *reinterpret_cast<DecompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
@@ -90,7 +96,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     const uint64_t hn = *reinterpret_cast<const uint64_t*>(h + 8);
     eb = *reinterpret_cast<const float*>(h + 16);
     const uint64_t pbytes = *reinterpret_cast<const uint64_t*>(h + 24);
-    if (magic != 0x505A5343u || h[4] != CUSZP_VERSION || h[7] != 5) err = CUSZP_ECORRUPT;
+    if (magic != 0x505A5343u || h[4] != CUSZP_VERSION || h[7] != kLog2L) err = CUSZP_ECORRUPT;
     else if (h[6] != CUSZP_OK) err = (h[6] == CUSZP_ERANGE) ? CUSZP_ERANGE : CUSZP_ECORRUPT;
     else if (hn != a.n) err = CUSZP_EINVAL;
     else if (a.n > 0) {
@@ -127,11 +133,25 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
         }
         const uint32_t t0 = c * kChunkTiles;
         const uint32_t ntiles = min(uint32_t(kChunkTiles), a.num_tiles - t0);
-        // lane L: blocks 16L .. 16L+15 of the chunk = groups 4(L%8) .. +3 of tile L/8
-        const uint64_t blk = uint64_t(t0) * kTileBlocks + 16u * lane;
-        uint4 fq = make_uint4(0, 0, 0, 0);
-        if (blk < a.nb) fq = *reinterpret_cast<const uint4*>(a.in + kHdr + blk);   // in the 16-B padded F area
-        const uint32_t fw[4] = {fq.x, fq.y, fq.z, fq.w};
+        // lane L: sub-blocks 16L .. 16L+15 of the chunk = groups 4(L%8) .. +3 of
+        // tile L/8 = blocks (16L .. 16L+15) / M
+        const uint64_t blk = (uint64_t(t0) * kTileBlocks + 16u * lane) / M;
+        uint32_t fw[4] = {0, 0, 0, 0};
+        if (blk < a.nb) {                                              // in the 16-B padded F area
+          if constexpr (M == 1) {
+            const uint4 fq = *reinterpret_cast<const uint4*>(a.in + kHdr + blk);
+            fw[0] = fq.x; fw[1] = fq.y; fw[2] = fq.z; fw[3] = fq.w;
+          } else if constexpr (M == 2) {
+            // F of blocks 2g, 2g+1 replicated onto sub-blocks (4g .. 4g+3)
+            const uint2 fq = *reinterpret_cast<const uint2*>(a.in + kHdr + blk);
+            fw[0] = __byte_perm(fq.x, 0, 0x1100u); fw[1] = __byte_perm(fq.x, 0, 0x3322u);
+            fw[2] = __byte_perm(fq.y, 0, 0x1100u); fw[3] = __byte_perm(fq.y, 0, 0x3322u);
+          } else {
+            const uint32_t fq = *reinterpret_cast<const uint32_t*>(a.in + kHdr + blk);
+            fw[0] = __byte_perm(fq, 0, 0x0000u); fw[1] = __byte_perm(fq, 0, 0x1111u);
+            fw[2] = __byte_perm(fq, 0, 0x2222u); fw[3] = __byte_perm(fq, 0, 0x3333u);
+          }
+        }
         uint32_t gw[4], gspan[4], gsum[4], lsum = 0;
 #pragma unroll
         for (int g = 0; g < 4; ++g) {
@@ -141,7 +161,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             uint32_t f = (fw[g] >> (8 * k)) & 0xffu;
-            if (blk + 4 * g + k >= a.nb) f = 0;
+            if (blk + (4 * g + k) / M >= a.nb) f = 0;
             if (f > uint32_t(kMaxF)) { bad |= kBadCorrupt; f = 0; }
             const uint32_t wq = f ? f + 1 : 0;             // Eq 2 in 4-byte words
             gw[g] |= wq << (8 * k);
@@ -280,7 +300,32 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           const uint32_t pbytes = wbytes * 0x01010100u;             // exclusive word prefix per block
           uint32_t sel, row;                                         // phase-2 source of this lane
           // a10: load each packed block's words into its lane range, one transpose per row
-          if (mode == 0) {
+          if (M > 1 && mode == 0) {
+            // word k8 of sub-block q at pre(block) + M k8 + q % M
+            const uint32_t wq = __byte_perm(wbytes, 0, sel_quad);
+            const uint32_t pq = __byte_perm(pbytes, 0, 0x4440u + (q & ~uint32_t(M - 1))) + M * k8 + (q & (M - 1));
+            scratch[lane] = xpose(k8 < wq ? gdata[pq] : 0u);
+            sel = sel_quad;
+            row = 0;
+          } else if (M > 1 && mode == 1) {
+            const uint32_t w0 = wbytes & 0xffu, w2 = (wbytes >> 16) & 0xffu;
+            const uint32_t h = hi ? 1u : 0u;
+            const uint32_t x01 = k16 < w0 ? gdata[M * k16 + h] : 0u;
+            const uint32_t x23 = k16 < w2 ? gdata[(M == 2 ? 2 * w0 : 0u) + M * k16 + (M == 2 ? h : 2u + h)] : 0u;
+            scratch[lane] = xpose(x01);
+            scratch[32 + lane] = xpose(x23);
+            sel = sel_pair;
+            row = row_pair;
+          } else if (M > 1) {
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+              const uint32_t wq = (wbytes >> (8 * b)) & 0xffu;
+              const uint32_t oq = ((pbytes >> (8 * (b & ~(M - 1)))) & 0xffu) + (b & (M - 1));
+              scratch[32 * b + lane] = xpose(uint32_t(lane) < wq ? gdata[oq + M * uint32_t(lane)] : 0u);
+            }
+            sel = 0x3210u;
+            row = row_single;
+          } else if (mode == 0) {
             const uint32_t wq = __byte_perm(wbytes, 0, sel_quad), pq = __byte_perm(pbytes, 0, sel_quad);
             scratch[lane] = xpose(k8 < wq ? gdata[pq + k8] : 0u);
             sel = sel_quad;
@@ -320,9 +365,12 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           e2 += e1;
           e3 += e2;
           int incl = e3;
-          incl = scan_step_up(incl, 1, 24 << 8);
-          incl = scan_step_up(incl, 2, 24 << 8);
-          incl = scan_step_up(incl, 4, 24 << 8);
+          constexpr int kSeg = (32 - 8 * M) << 8;                     // segment = the block's 8 M lanes
+          incl = scan_step_up(incl, 1, kSeg);
+          incl = scan_step_up(incl, 2, kSeg);
+          incl = scan_step_up(incl, 4, kSeg);
+          if constexpr (M >= 2) incl = scan_step_up(incl, 8, kSeg);
+          if constexpr (M >= 4) incl = scan_step_up(incl, 16, kSeg);
           const int carry = incl - e3;
           // a12: d' = r * 2eb
           float4 d;
@@ -362,6 +410,10 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     finish_call(a.ws, a.status, a.status_cap, epoch, final_status);
   }
 }
+
+template __global__ void decompress_kernel<1>(DecompressArgs);
+template __global__ void decompress_kernel<2>(DecompressArgs);
+template __global__ void decompress_kernel<4>(DecompressArgs);
 
 size_t decompress_smem_bytes() { return sizeof(DecompressSmem); }
 int decompress_threads() { return kDThreads; }

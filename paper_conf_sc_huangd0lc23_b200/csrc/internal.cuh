@@ -420,9 +420,9 @@ struct QualityArgs {
 };
 constexpr int kQualityMaxGrid = 2048;
 
-__global__ void compress_kernel(CompressArgs a);
+template <int M> __global__ void compress_kernel(CompressArgs a);      // M = L / 32
 __global__ void quality_kernel(QualityArgs a);
-__global__ void decompress_kernel(DecompressArgs a);
+template <int M> __global__ void decompress_kernel(DecompressArgs a);
 __global__ void range_kernel(RangeArgs a);
 int launch_copy_len(void* dst, const void* src, const unsigned long long* d_len, uint64_t cap,
                     unsigned long long* len_out, int sms, cudaStream_t s);

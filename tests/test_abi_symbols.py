@@ -97,3 +97,11 @@ def test_binding_rejects_cpu_tensors():
 
     with pytest.raises(TypeError):
         cz.compress(torch.zeros(10), 1e-3)
+
+
+def test_max_compressed_bytes_L_matches_oracle():
+    h = _lib.lib()
+    for Lb in (32, 64, 128):
+        for n in (0, 1, 2, 31, 64, 129, 10**6 + 3):
+            assert h.cuszp_max_compressed_bytes_L(n, Lb) == oracle.max_compressed_bytes_L(n, Lb)
+    assert h.cuszp_max_compressed_bytes_L(100, 48) == 0

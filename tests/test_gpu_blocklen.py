@@ -1,0 +1,76 @@
+"""GPU parity of the block-length variants L in {64, 128} (SURVEY 8(f) NEXT
+rank 3) against oracle.compress_L / oracle.decompress: compressed bytes
+identical, decompressed floats bit-identical, on sizes spanning many tiles
+with ragged tails and on fields that exercise all three packing modes of
+the kernels (F <= 7, F <= 15, F up to 24)."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_sc_huangd0lc23_b200 as cz
+import synth
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda"
+
+
+def parity(x_np: np.ndarray, eb: float, mode: int, Lb: int, label=""):
+    x = torch.from_numpy(x_np).to(DEV)
+    st_o, s_o = oracle.compress_L(x_np, eb, mode, Lb)
+    out, nb = cz.compress(x, eb, mode, block_len=Lb)
+    torch.cuda.synchronize()
+    s_g = out[: int(nb.item())].cpu().numpy()
+    assert s_g[6] == st_o, (label, s_g[6], st_o)
+    if st_o != oracle.OK:
+        return
+    assert s_g.size == s_o.size, (label, s_g.size, s_o.size)
+    if not np.array_equal(s_g, s_o):
+        bad = np.nonzero(s_g != s_o)[0]
+        raise AssertionError(f"{label}: {bad.size} bytes differ, first at {bad[0]} of {s_o.size}")
+    st, y_o = oracle.decompress(s_o, x_np.size)
+    y = cz.decompress(out, x_np.size, in_bytes=s_o.size, block_len=Lb)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32)), label
+
+
+@pytest.mark.parametrize("Lb", [64, 128])
+@pytest.mark.parametrize("n", [2, 31, 64, 65, 129, 4096, 4097, 100_003, 1 << 20])
+def test_sizes(Lb, n):
+    rng = np.random.default_rng(n)
+    x = np.cumsum(rng.standard_normal(n)).astype(np.float32)
+    x[n // 3: n // 2] = 0.0
+    parity(x, 1e-3, oracle.REL, Lb, f"L={Lb} n={n}")
+
+
+@pytest.mark.parametrize("Lb", [64, 128])
+@pytest.mark.parametrize("field,rel", [("U", 1e-2), ("QCLOUD", 1e-3), ("TC", 1e-4)])
+def test_hurricane_fields(Lb, field, rel):
+    x = synth.hurricane_like(field, shape=(20, 100, 100), device="cpu").numpy()
+    parity(x, rel, oracle.REL, Lb, f"L={Lb} {field}@{rel}")
+
+
+@pytest.mark.parametrize("Lb", [64, 128])
+def test_wide_fixed_lengths(Lb):
+    # ABS with a tiny bound: F up to the guard's 24 bits (one block per transpose)
+    rng = np.random.default_rng(Lb)
+    x = (rng.standard_normal(300_000) * 1e3).astype(np.float32)
+    for eb in (1e-3, 1.0, 30.0):
+        parity(x, eb, oracle.ABS, Lb, f"L={Lb} abs eb={eb}")
+
+
+@pytest.mark.parametrize("Lb", [64, 128])
+def test_minmax_and_wrong_L(Lb):
+    x_np = synth.smooth1d(200_000, seed=3, device="cpu").numpy()
+    x = torch.from_numpy(x_np).to(DEV)
+    mm = torch.tensor([-5.0, 7.0], device=DEV)
+    st, s_o = oracle.compress_minmax_L(x_np, 1e-4, mm.cpu().numpy(), Lb)
+    out, nb = cz.compress_minmax(x, 1e-4, mm, block_len=Lb)
+    torch.cuda.synchronize()
+    assert np.array_equal(out[: int(nb.item())].cpu().numpy(), s_o)
+    cz.decompress(out, x.numel(), block_len=32)          # header says another L
+    assert cz.last_status() == cz.ECORRUPT
+    with pytest.raises(cz.CuszpError):
+        cz.compress(x, 1e-3, "rel", block_len=48)

@@ -184,6 +184,8 @@ def test_fuzzed_streams_never_fault():
     x = torch.from_numpy(rng.standard_normal(70_000).astype(np.float32)).to(DEV)
     out, nb = cz.compress(x, 1e-3, "rel")
     n = int(nb.item())
+    assert cz.read_header(out)["status"] == cz.OK, cz.read_header(out)
+    assert n > 32 + 2200 + 16, n
     base = out[:n].clone()
     ws = cz.Workspace(70_000)
     y = torch.empty(70_000, device=DEV)
@@ -299,3 +301,21 @@ def test_full_size_rtm_sampled():
         ax = xs.abs()
         ulp = torch.nextafter(ax.float(), torch.full_like(ax.float(), float("inf"))).double() - ax
         assert bool(((ys - xs).abs() <= float(eb) + ulp).all())
+
+
+@pytest.mark.parametrize("Lb", [32, 64, 128])
+def test_guard_failures_never_write_past_capacity(Lb):
+    """Data failing the R5 guard (|x/2eb| >= 2^22, NaN, Inf) encode garbage
+    blocks before the status is known: the kernel must still stay inside
+    cuszp_max_compressed_bytes_L(n, L) (a canary after the buffer)."""
+    n = 1000
+    cap = cz.max_compressed_bytes(n, Lb)
+    for x in (torch.arange(n, dtype=torch.float32, device=DEV) * 1e6,
+              torch.full((n,), float("inf"), device=DEV),
+              torch.full((n,), float("nan"), device=DEV)):
+        buf = torch.full((cap + 4096,), 0xA5, dtype=torch.uint8, device=DEV)
+        out_bytes = torch.zeros(1, dtype=torch.int64, device=DEV)
+        cz.compress(x, 1e-9, "abs", out=buf[:cap], out_bytes=out_bytes, block_len=Lb)
+        torch.cuda.synchronize()
+        assert cz.read_header(buf)["status"] == cz.ERANGE
+        assert bool((buf[cap:] == 0xA5).all()), "wrote past the capacity"
