@@ -317,6 +317,41 @@ def run_ours(args, rank, world, dev):
     q_bytes = sum(8 * n_of[f] for f, _ in jobs)
     quality["kernel_gbs"] = q_bytes / (sum(q_ms) / 1e3) / 1e9
 
+    # block-length variants on the first field at the
+    # middle bound: compress and decompress kernels, L2 flushed, median of 5
+    f0, rel0 = fields[0], rels[len(rels) // 2]
+    x0, n0 = xs[f0], n_of[f0]
+    cz.check(lib.cuszp_range(x0.data_ptr(), n0, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
+    variants = {}
+    for Lb in (32, 64, 128):
+        tc, td = [], []
+        capL = cz.max_compressed_bytes(n0, Lb)
+        outL = out if capL <= cap else torch.empty(capL, dtype=torch.uint8, device=dev)
+        for _ in range(6):
+            flush_l2()
+            qev[0].record(stream)
+            cz.check(lib.cuszp_compress_minmax_L(x0.data_ptr(), n0, float(rel0), mm_local.data_ptr(), 1, Lb,
+                                                 outL.data_ptr(), capL, out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
+                                                 sp), "compress_L")
+            qev[1].record(stream)
+            torch.cuda.synchronize(dev)
+            tc.append(qev[0].elapsed_time(qev[1]))
+            flush_l2()
+            qev[0].record(stream)
+            cz.check(lib.cuszp_decompress_L(outL.data_ptr(), capL, y.data_ptr(), n0, Lb, ws.ptr(), ws.nbytes, sp),
+                     "decompress_L")
+            qev[1].record(stream)
+            torch.cuda.synchronize(dev)
+            td.append(qev[0].elapsed_time(qev[1]))
+        assert cz.last_status(ws) == cz.OK
+        SL = int(out_bytes.item())
+        tcm, tdm = float(np.median(tc[1:])) / 1e3, float(np.median(td[1:])) / 1e3
+        variants[str(Lb)] = {"cr": round(4 * n0 / SL, 3),
+                             "compress_kernel_gbs": round(4 * n0 / tcm / 1e9, 1),
+                             "decompress_kernel_gbs": round(4 * n0 / tdm / 1e9, 1),
+                             "compress_frac_of_peak": round((4 * n0 + SL) / tcm / 1e9 / peak_hbm()[0], 4),
+                             "decompress_frac_of_peak": round((4 * n0 + SL) / tdm / 1e9 / peak_hbm()[0], 4)}
+
     t_dev = torch.tensor([acc["range"], acc["compress"], acc["decompress"]], dtype=torch.float64, device=dev)
     if world > 1:
         torch.distributed.all_reduce(t_dev, op=torch.distributed.ReduceOp.MAX)
@@ -363,6 +398,7 @@ def run_ours(args, rank, world, dev):
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
         "gpu_launches": 3 * len(jobs) * K,
+        "block_len_variants": {"workload": f"{f0}@{rel0:g}", "unit": "GB/s of fp32 input", **variants},
         "quality": dict(quality, frac_of_peak=quality["kernel_gbs"] / peak,
                         kernel="cuszp_quality (fused compareData statistics, untimed verification pass)"),
         "clocks": clk,
