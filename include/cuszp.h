@@ -66,9 +66,11 @@ typedef struct {
   uint64_t payload_bytes;  /* sum of CmpL_k (Eq 2, Eq 3 total) */
 } cuszp_header;
 
-/* Largest stream for n elements: 32 + align16(ceil(n/32)) + 100*ceil(n/32)
- * (F <= 24 by the R5 guard, so CmpL <= 4*25).  Output buffers of compress
- * must be at least this large. */
+/* Output buffer size for n elements: 32 + align16(nb) + 128*nb, nb =
+ * ceil(n/32).  A valid stream is at most 32 + align16(nb) + 100*nb (F <= 24
+ * by the R5 guard, CmpL <= 4*25); data that fail the guard are only known to
+ * be ERANGE at the end of the kernel and may have written up to 32 words per
+ * block by then.  Output buffers of compress must be at least this large. */
 size_t cuszp_max_compressed_bytes(size_t n);
 
 /* Exact compressed size from the per-block fixed lengths F[0..nb) (host
@@ -123,7 +125,7 @@ int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n,
  * bit j%8 (R9 generalised); header byte 7 = log2(L); one F byte
  * per L-block.  The calls without _L are the L = 32 ones.  Output buffers
  * need cuszp_max_compressed_bytes_L(n, L) bytes (32 + align16(nb) +
- * 25 L/8 nb, nb = ceil(n/L)); workspaces are sized as for L = 32.
+ * 32 L/8 nb, nb = ceil(n/L)); workspaces are sized as for L = 32.
  * block_len outside {32, 64, 128}: EINVAL (the size helper returns 0).
  * Decompression must be given the stream's L (a header with another L:
  * async ECORRUPT). */

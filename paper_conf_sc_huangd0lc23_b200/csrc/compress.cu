@@ -58,7 +58,7 @@ constexpr int kFirstCompute = 1 + kWriters;
 constexpr int kTix = 16;                          // ticket ring: producer -> writers (early look-back)
 static_assert(kStages + kMeta + kWriters <= kTix, "ticket ring");
 constexpr int kCThreads = (kFirstCompute + kComputeWarps) * 32;
-static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * kMaxBlockWords, "ring size");
+static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * 32, "ring size");
 
 struct TileMeta {
   uint32_t tile;
@@ -345,8 +345,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               v[q] = lorenzo_pack_first(r[q], lane,
                                         (q % M == 0) ? kRoundMagicBits : __shfl_sync(kFull, r[q > 0 ? q - 1 : 0], 31));
           }
-          // room in this warp's ring for a worst-case group (4 x 25 words)
-          while (head + cursor + 4 * kMaxBlockWords - ld_volatile_u32(&sm.tail[w]) > kRing)
+          // room in this warp's ring for a worst-case group (4 x 32 words)
+          while (head + cursor + 4 * 32 - ld_volatile_u32(&sm.tail[w]) > kRing)
             __nanosleep(CUSZP_C_POLL_NS);
 #ifdef CUSZP_DIAG_TINY
           v[0] = v[1] = v[2] = v[3] = 0;   // diagnostics only: all zero blocks (wrong output)
@@ -359,19 +359,17 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(__reduce_or_sync(kFull, v[q])));   // -1 for 0
             wq[q] = b + 1;
           }
-          // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
-          // record it, and clamp so an ERANGE stream never exceeds the
-          // capacity bound (25 words per block) nor the ring reservation
-          wmax = max(wmax, max(max(wq[0], wq[1]), max(wq[2], wq[3])));
-#pragma unroll
-          for (int q = 0; q < 4; ++q) wq[q] = min(wq[q], uint32_t(kMaxBlockWords));
           if constexpr (M == 2) {                                        // one F per block
             wq[0] = wq[1] = max(wq[0], wq[1]);
             wq[2] = wq[3] = max(wq[2], wq[3]);
           } else if constexpr (M == 4) {
             wq[0] = wq[1] = wq[2] = wq[3] = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
           }
+          // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
+          // flagged ERANGE at the end.  Such garbage blocks still take at most
+          // 32 words (v is 32-bit), which the capacity bound covers (DESIGN 9.5).
           const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+          wmax = max(wmax, span);
           const uint32_t wb = wq[0] | (wq[1] << 8) | (wq[2] << 16) | (wq[3] << 24);
           const uint32_t base = head + cursor;
           if (M > 1) {

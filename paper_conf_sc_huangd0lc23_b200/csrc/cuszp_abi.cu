@@ -118,8 +118,11 @@ size_t cuszp_max_compressed_bytes(size_t n) { return cuszp_max_compressed_bytes_
 
 size_t cuszp_max_compressed_bytes_L(size_t n, int block_len) {
   if (sub_blocks(block_len) == 0) return 0;
+  // a valid block takes at most 25 words (F <= 24, R5); a block of data that
+  // fails the guard is only known to be ERANGE at the end of the kernel and
+  // may take 32 (v is 32-bit): the bound covers that too (DESIGN 9.5)
   const uint64_t nb = num_blocks(n, block_len);
-  return size_t(kHdr + align16(nb) + uint64_t(block_len / 8) * (kMaxF + 1) * nb);
+  return size_t(kHdr + align16(nb) + uint64_t(block_len / 8) * 32u * nb);
 }
 
 size_t cuszp_compressed_bytes_from_F(const uint8_t* h_F, size_t nb) {

@@ -41,7 +41,7 @@ def main():
     libs = [load(p) for p in a.libs]
     h0 = libs[0]
     ws = torch.zeros(max(l.cuszp_workspace_bytes(n) for l in libs), dtype=torch.uint8, device=dev)
-    cap = h0.cuszp_max_compressed_bytes(n)
+    cap = max(l.cuszp_max_compressed_bytes(n) for l in libs)
     out = torch.empty(cap, dtype=torch.uint8, device=dev)
     ob = torch.zeros(1, dtype=torch.int64, device=dev)
     mm = torch.empty(2, dtype=torch.float32, device=dev)
