@@ -496,9 +496,27 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   }
 }
 
-template __global__ void compress_kernel<1>(CompressArgs);
-template __global__ void compress_kernel<2>(CompressArgs);
-template __global__ void compress_kernel<4>(CompressArgs);
+namespace {
+template <int M>
+cudaError_t configure_m(int* occ) {
+  const int smem = int(sizeof(CompressSmem));
+  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M>, kCThreads, smem);
+  return e;
+}
+}  // namespace
+
+cudaError_t compress_configure(int M, int* occ) {
+  return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
+}
+
+cudaError_t compress_launch(int M, unsigned grid, const CompressArgs& a, cudaStream_t s) {
+  const size_t smem = sizeof(CompressSmem);
+  if (M == 1) compress_kernel<1><<<grid, kCThreads, smem, s>>>(a);
+  else if (M == 2) compress_kernel<2><<<grid, kCThreads, smem, s>>>(a);
+  else compress_kernel<4><<<grid, kCThreads, smem, s>>>(a);
+  return cudaGetLastError();
+}
 
 size_t compress_smem_bytes() { return sizeof(CompressSmem); }
 int compress_threads() { return kCThreads; }

@@ -34,22 +34,13 @@ int device_info(DeviceInfo* out) {
   std::lock_guard<std::mutex> lock(mu);
   if (!have[dev]) {
     DeviceInfo d;
-    const int cs = int(compress_smem_bytes()), ds = int(decompress_smem_bytes());
-    if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
-        cudaFuncSetAttribute(compress_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
-        cudaFuncSetAttribute(compress_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
-        cudaFuncSetAttribute(compress_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, cs) != cudaSuccess ||
-        cudaFuncSetAttribute(decompress_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess ||
-        cudaFuncSetAttribute(decompress_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess ||
-        cudaFuncSetAttribute(decompress_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, ds) != cudaSuccess)
-      return CUSZP_ECUDA;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_c[0], compress_kernel<1>, compress_threads(), cs) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_c[1], compress_kernel<2>, compress_threads(), cs) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_c[2], compress_kernel<4>, compress_threads(), cs) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_d[0], decompress_kernel<1>, decompress_threads(), ds) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_d[1], decompress_kernel<2>, decompress_threads(), ds) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_d[2], decompress_kernel<4>, decompress_threads(), ds) != cudaSuccess ||
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess ||
+    if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return CUSZP_ECUDA;
+    for (int k = 0; k < 3; ++k) {
+      const int M = 1 << k;
+      if (compress_configure(M, &d.occ_c[k]) != cudaSuccess || decompress_configure(M, &d.occ_d[k]) != cudaSuccess)
+        return CUSZP_ECUDA;
+    }
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_quality, quality_kernel, 256, 0) != cudaSuccess)
       return CUSZP_ECUDA;
     d.occ_compress = d.occ_c[0];
@@ -104,10 +95,7 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  if (M == 1) compress_kernel<1><<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
-  else if (M == 2) compress_kernel<2><<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
-  else compress_kernel<4><<<unsigned(grid), compress_threads(), compress_smem_bytes(), stream>>>(a);
-  return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+  return compress_launch(M, unsigned(grid), a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
 }  // namespace
@@ -260,10 +248,7 @@ int cuszp_decompress_L(const void* d_in, size_t in_bytes, float* d_out, size_t n
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  if (M == 1) decompress_kernel<1><<<unsigned(grid), decompress_threads(), decompress_smem_bytes(), s>>>(a);
-  else if (M == 2) decompress_kernel<2><<<unsigned(grid), decompress_threads(), decompress_smem_bytes(), s>>>(a);
-  else decompress_kernel<4><<<unsigned(grid), decompress_threads(), decompress_smem_bytes(), s>>>(a);
-  return cudaGetLastError() == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+  return decompress_launch(M, unsigned(grid), a, s) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
 int cuszp_last_status(const void* d_ws, void* stream) {

@@ -411,9 +411,27 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
   }
 }
 
-template __global__ void decompress_kernel<1>(DecompressArgs);
-template __global__ void decompress_kernel<2>(DecompressArgs);
-template __global__ void decompress_kernel<4>(DecompressArgs);
+namespace {
+template <int M>
+cudaError_t configure_m(int* occ) {
+  const int smem = int(sizeof(DecompressSmem));
+  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M>, kDThreads, smem);
+  return e;
+}
+}  // namespace
+
+cudaError_t decompress_configure(int M, int* occ) {
+  return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
+}
+
+cudaError_t decompress_launch(int M, unsigned grid, const DecompressArgs& a, cudaStream_t s) {
+  const size_t smem = sizeof(DecompressSmem);
+  if (M == 1) decompress_kernel<1><<<grid, kDThreads, smem, s>>>(a);
+  else if (M == 2) decompress_kernel<2><<<grid, kDThreads, smem, s>>>(a);
+  else decompress_kernel<4><<<grid, kDThreads, smem, s>>>(a);
+  return cudaGetLastError();
+}
 
 size_t decompress_smem_bytes() { return sizeof(DecompressSmem); }
 int decompress_threads() { return kDThreads; }
