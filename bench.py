@@ -493,11 +493,17 @@ def main():
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
-    dev = torch.device("cuda", local)
+    # CUSZP_BENCH_SHARE_GPU=1 (diagnostics only): every rank on the same GPU
+    # over gloo, to exercise the N > 1 code path on a one-GPU box
+    share = os.environ.get("CUSZP_BENCH_SHARE_GPU") == "1"
+    dev = torch.device("cuda", local % torch.cuda.device_count() if share else local)
     torch.cuda.set_device(dev)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        torch.distributed.init_process_group("nccl", device_id=dev)
+        if share:
+            torch.distributed.init_process_group("gloo")
+        else:
+            torch.distributed.init_process_group("nccl", device_id=dev)
     line = run_ours(args, rank, world, dev)
     if rank == 0:
         print(json.dumps(line), flush=True)
