@@ -245,7 +245,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         // prefix matters: do not poll predecessors that early
         __nanosleep(CUSZP_C_LB_DELAY);
 #endif
+#ifdef CUSZP_TRACE
         const uint64_t t_lb = a.trace ? global_ns() : 0;
+#endif
         const uint64_t excl = resolve_excl(a.status, t, epoch, &nw, &ns);
         mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
         const TileMeta& md = sm.meta[m];
@@ -259,12 +261,14 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           const uint32_t y = __shfl_up_sync(kFull, incl, o);
           if (lane >= o) incl += y;
         }
+#ifdef CUSZP_TRACE
         if (lane == 0 && a.trace) {
           trace_put(a.trace, t, 3, t_lb);
           trace_put(a.trace, t, 4, global_ns());
           trace_put(a.trace, t, 5, nw);
           trace_put(a.trace, t, 6, ns);
         }
+#endif
         // a8 store: each compute warp's ring segment -> [excl + warp offset, ...)
 #pragma unroll 1
         for (int w = 0; w < kComputeWarps; ++w) {
@@ -296,10 +300,17 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const int m = int(i % kMeta);
         mbar_wait(&sm.full[s], (i / kStages) & 1u);         // suspending wait: no issue slots taken
         const uint32_t t = sm.in_tile[s];
+#ifdef CUSZP_TRACE
+        // (diagnostics build only: a lane-0 branch here makes ptxas treat the
+        // whole encode as possibly divergent -- a divergence check before every
+        // warp-synchronous op and 60 % more code)
         if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 7, global_ns());
+#endif
         // meta slot m free (tile i - kMeta released)
         while (int(i - ld_volatile_u32(&sm.released)) >= kMeta) __nanosleep(CUSZP_C_POLL_NS);
+#ifdef CUSZP_TRACE
         if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
+#endif
         if (t == kSentinel) break;                    // the writers stop on the ticket ring
         const bool last = (t == a.num_tiles - 1);
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;   // first element of the warp

@@ -2,6 +2,11 @@
 
     python tools/trace_scan.py [--lib path/to/libcuszp_variant.so] [--config c2_hurricane]
 
+Needs a library built with -DCUSZP_TRACE (the production build compiles the
+compute-warp trace points out: a lane-0 branch in the encode loop costs ~6 %):
+    python tools/build_variants.py trace:CUSZP_TRACE
+    python tools/trace_scan.py --lib build_variants/trace.so
+
 Installs a trace buffer (cuszp_debug_set_trace), runs range + compress +
 decompress on one field and prints, per kernel, the distribution of the
 per-tile phases recorded with %globaltimer:
