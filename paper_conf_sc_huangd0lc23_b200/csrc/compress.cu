@@ -144,6 +144,11 @@ __device__ __forceinline__ uint32_t lorenzo_pack_first(uint32_t rb, int lane, ui
   return (a << 1) | (uint32_t(l) >> 31);
 }
 
+// bytes a, b, c, d (each < 256) -> one word, as 3 byte permutes
+__device__ __forceinline__ uint32_t pack4(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  return __byte_perm(__byte_perm(a, b, 0x3240u), __byte_perm(c, d, 0x3240u), 0x5410u);
+}
+
 }  // namespace
 
 // M = L / 32: an L-block is M consecutive 32-element
@@ -381,19 +386,19 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           // 32 words (v is 32-bit), which the capacity bound covers (DESIGN 9.5).
           const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
           wmax = max(wmax, span);
-          const uint32_t wb = wq[0] | (wq[1] << 8) | (wq[2] << 16) | (wq[3] << 24);
+          const uint32_t wb = pack4(wq[0], wq[1], wq[2], wq[3]);
           const uint32_t base = head + cursor;
           if (M > 1) {
             // word k of sub-block q -> block payload position M k + q % M
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
             if (span <= 8) {
-              const uint32_t tw = xpose(v[0] | (v[1] << 8) | (v[2] << 16) | (v[3] << 24));
+              const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
               const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
               const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
               if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;
             } else if (span <= 16) {
-              const uint32_t t01 = xpose(v[0] | (v[1] << 16));
-              const uint32_t t23 = xpose(v[2] | (v[3] << 16));
+              const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
+              const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
               const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
               if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;
               const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
@@ -408,13 +413,13 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               }
             }
           } else if (span <= 8) {
-            const uint32_t tw = xpose(v[0] | (v[1] << 8) | (v[2] << 16) | (v[3] << 24));
+            const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
             const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
             if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;
           } else if (span <= 16) {
-            const uint32_t t01 = xpose(v[0] | (v[1] << 16));
-            const uint32_t t23 = xpose(v[2] | (v[3] << 16));
+            const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
+            const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
             const bool hi = lane >= 16;
             const uint32_t k = lane & 15;
             if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;
