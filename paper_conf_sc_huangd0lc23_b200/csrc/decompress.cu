@@ -27,10 +27,10 @@ namespace cuszp {
 namespace {
 
 #ifndef CUSZP_D_MINBLOCKS
-#define CUSZP_D_MINBLOCKS 3
+#define CUSZP_D_MINBLOCKS 4   // 4 CTAs x 10 warps per SM: the decode is latency-bound (48 registers, no spills)
 #endif
 #ifndef CUSZP_D_STAGES
-#define CUSZP_D_STAGES 4
+#define CUSZP_D_STAGES 2
 #endif
 constexpr int kDStages = CUSZP_D_STAGES;
 #ifndef CUSZP_D_UNROLL
