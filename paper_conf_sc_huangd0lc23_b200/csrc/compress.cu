@@ -162,6 +162,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
   const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);   // provably warp-uniform (no divergence checks before warp-sync ops)
+  pdl_wait();                                     // range kernel / previous call complete
+  pdl_launch_dependents();
   const uint32_t epoch = running_epoch(a.ws);
 
   // ---- eb_abs (Eq 1): ABS -> delta; REL -> lambda * (max - min) over the (min,max) pairs
@@ -527,11 +529,19 @@ cudaError_t compress_configure(int M, int* occ) {
 }
 
 cudaError_t compress_launch(int M, unsigned grid, const CompressArgs& a, cudaStream_t s) {
-  const size_t smem = sizeof(CompressSmem);
-  if (M == 1) compress_kernel<1><<<grid, kCThreads, smem, s>>>(a);
-  else if (M == 2) compress_kernel<2><<<grid, kCThreads, smem, s>>>(a);
-  else compress_kernel<4><<<grid, kCThreads, smem, s>>>(a);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kCThreads);
+  cfg.dynamicSmemBytes = sizeof(CompressSmem);
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;   // see pdl_wait()
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (M == 1) return cudaLaunchKernelEx(&cfg, compress_kernel<1>, a);
+  if (M == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<2>, a);
+  return cudaLaunchKernelEx(&cfg, compress_kernel<4>, a);
 }
 
 size_t compress_smem_bytes() { return sizeof(CompressSmem); }

@@ -81,6 +81,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
   DecompressSmem& sm = *reinterpret_cast<DecompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
+  pdl_wait();                                     // compression / previous call complete
   const uint32_t epoch = running_epoch(a.ws);
 
   // ---- header (R10), validated identically by every thread
@@ -426,11 +427,19 @@ cudaError_t decompress_configure(int M, int* occ) {
 }
 
 cudaError_t decompress_launch(int M, unsigned grid, const DecompressArgs& a, cudaStream_t s) {
-  const size_t smem = sizeof(DecompressSmem);
-  if (M == 1) decompress_kernel<1><<<grid, kDThreads, smem, s>>>(a);
-  else if (M == 2) decompress_kernel<2><<<grid, kDThreads, smem, s>>>(a);
-  else decompress_kernel<4><<<grid, kDThreads, smem, s>>>(a);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kDThreads);
+  cfg.dynamicSmemBytes = sizeof(DecompressSmem);
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;   // see pdl_wait()
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (M == 1) return cudaLaunchKernelEx(&cfg, decompress_kernel<1>, a);
+  if (M == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<2>, a);
+  return cudaLaunchKernelEx(&cfg, decompress_kernel<4>, a);
 }
 
 size_t decompress_smem_bytes() { return sizeof(DecompressSmem); }

@@ -204,6 +204,14 @@ struct Xpose {
   }
 };
 
+// --------------------------------------------- programmatic dependent launch
+// The scan kernels are launched with programmatic stream serialisation: their
+// CTAs may be scheduled while the previous kernel's CTAs retire, and wait here
+// (before touching anything that kernel wrote) for its completion and memory.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// Lets the next (PDL-launched) kernel be scheduled as this grid's CTAs retire.
+__device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" :::); }
+
 // ------------------------------------------------------------- diagnostics
 __device__ __forceinline__ uint64_t global_ns() {
   uint64_t t;

@@ -27,6 +27,7 @@ __device__ __forceinline__ float key_to_float(uint32_t k) {
 }  // namespace
 
 __global__ void __launch_bounds__(256) range_kernel(RangeArgs a) {
+  pdl_launch_dependents();   // the compression kernel may be scheduled as these CTAs retire
   uint32_t kmax = 0u;          // max key
   uint32_t kmin = 0xffffffffu; // min key
   const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;

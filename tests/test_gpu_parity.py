@@ -319,3 +319,34 @@ def test_guard_failures_never_write_past_capacity(Lb):
         torch.cuda.synchronize()
         assert cz.read_header(buf)["status"] == cz.ERANGE
         assert bool((buf[cap:] == 0xA5).all()), "wrote past the capacity"
+
+
+def test_cuda_graph_capture_and_replay():
+    """The device calls never allocate or synchronise: range + compress +
+    decompress (launched with programmatic dependent launch) capture into a
+    CUDA graph whose replays reproduce the eager bytes and floats."""
+    x_np = synth.smooth1d(300_000, seed=4, device="cpu").numpy()
+    x = torch.from_numpy(x_np).to(DEV)
+    n = x.numel()
+    ws = cz.Workspace(n)
+    out = torch.empty(cz.max_compressed_bytes(n), dtype=torch.uint8, device=DEV)
+    nb = torch.zeros(1, dtype=torch.int64, device=DEV)
+    y = torch.empty(n, device=DEV)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):                      # warm-up outside capture (library init)
+        cz.compress(x, 1e-4, "rel", out=out, out_bytes=nb, ws=ws, stream=s)
+        cz.decompress(out, n, out=y, ws=ws, stream=s)
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        cz.compress(x, 1e-4, "rel", out=out, out_bytes=nb, ws=ws, stream=s)
+        cz.decompress(out, n, out=y, ws=ws, stream=s)
+    st, s_o = oracle.compress(x_np, 1e-4, oracle.REL)
+    st, y_o = oracle.decompress(s_o, n)
+    for _ in range(3):
+        out.zero_(); y.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert int(nb.item()) == s_o.size
+        assert np.array_equal(out[: s_o.size].cpu().numpy(), s_o)
+        assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32))
