@@ -428,7 +428,7 @@ def run_ours(args, rank, world, dev):
     if not args.no_e2e:
         h_in = {f: xs[f].cpu().pin_memory() for f in fields}
         lanes = []
-        n_lanes = 3
+        n_lanes = int(os.environ.get("CUSZP_E2E_LANES", "3"))
         for _ in range(n_lanes):
             lanes.append(dict(stream=torch.cuda.Stream(dev),
                               h_out=torch.zeros(cap, dtype=torch.uint8).pin_memory(),
