@@ -47,8 +47,11 @@ namespace {
 #ifndef CUSZP_C_LB_DELAY
 #define CUSZP_C_LB_DELAY 1500   // ns before a writer's first look-back poll (tile still loading/encoding)
 #endif
+#ifndef CUSZP_C_CW
+#define CUSZP_C_CW 8            // compute warps per CTA (each encodes 128 / CW blocks of a tile)
+#endif
 #ifndef CUSZP_C_MINBLOCKS
-#define CUSZP_C_MINBLOCKS 3
+#define CUSZP_C_MINBLOCKS (CUSZP_C_CW > 8 ? 2 : 3)
 #endif
 constexpr int kStages = CUSZP_C_STAGES;          // input ring depth (16 KB tiles)
 constexpr int kWriters = CUSZP_C_WRITERS;        // scan + writer warps
@@ -57,23 +60,26 @@ constexpr uint32_t kRing = CUSZP_C_RING_WORDS;   // words per compute-warp ring 
 constexpr int kFirstCompute = 1 + kWriters;
 constexpr int kTix = 16;                          // ticket ring: producer -> writers (early look-back)
 static_assert(kStages + kMeta + kWriters <= kTix, "ticket ring");
-constexpr int kCThreads = (kFirstCompute + kComputeWarps) * 32;
+constexpr int kCW = CUSZP_C_CW;                   // compute warps of this kernel
+constexpr int kCBPW = kTileBlocks / kCW;          // 32-element blocks per compute warp per tile
+static_assert(kCW == 8 || kCW == 16, "compute warps");
+constexpr int kCThreads = (kFirstCompute + kCW) * 32;
 static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * 32, "ring size");
 
 struct TileMeta {
   uint32_t tile;
   uint32_t agg;                    // words of the tile
-  uint16_t cnt[kComputeWarps];     // words per compute warp
-  uint16_t head[kComputeWarps];    // ring position of each warp's first word
+  uint16_t cnt[kCW];               // words per compute warp
+  uint16_t head[kCW];              // ring position of each warp's first word
 };
 
 struct CompressSmem {
   float in[kStages][kTileElems];                 // 48 KB
-  uint32_t ring[kComputeWarps][kRing];           // 32 KB
+  uint32_t ring[kCW][kRing];                     // 4 KB per compute warp
   TileMeta meta[kMeta];
   uint32_t in_tile[kStages];
   uint32_t meta_done[kMeta];
-  uint32_t tail[kComputeWarps];                  // ring words released (monotonic)
+  uint32_t tail[kCW];                            // ring words released (monotonic)
   uint32_t released;                             // CTA-local tiles released (monotonic)
   uint32_t tix[kTix];                            // tile of CTA-local tile j (slot j % kTix)
   uint64_t full[kStages], empty[kStages], staged[kMeta], tixbar[kTix];
@@ -191,10 +197,10 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   uint32_t* payload = reinterpret_cast<uint32_t*>(a.out + p0);
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kComputeWarps); }
+    for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kCW); }
     for (int m = 0; m < kMeta; ++m) { mbar_init(&sm.staged[m], 1); sm.meta_done[m] = 0; }
     for (int k = 0; k < kTix; ++k) mbar_init(&sm.tixbar[k], 1);
-    for (int w = 0; w < kComputeWarps; ++w) sm.tail[w] = 0;
+    for (int w = 0; w < kCW; ++w) sm.tail[w] = 0;
     sm.released = 0;
     fence_mbar_init();
   }
@@ -260,11 +266,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const TileMeta& md = sm.meta[m];
         const uint32_t agg = md.agg;
         if (lane == 0 && t > 0) publish_prefix(a.status, t, excl + agg, epoch);
-        const uint32_t cnt = lane < kComputeWarps ? md.cnt[lane] : 0u;
-        const uint32_t hd = lane < kComputeWarps ? md.head[lane] : 0u;
+        const uint32_t cnt = lane < kCW ? md.cnt[lane] : 0u;
+        const uint32_t hd = lane < kCW ? md.head[lane] : 0u;
         uint32_t incl = cnt;
 #pragma unroll
-        for (int o = 1; o < kComputeWarps; o <<= 1) {
+        for (int o = 1; o < kCW; o <<= 1) {
           const uint32_t y = __shfl_up_sync(kFull, incl, o);
           if (lane >= o) incl += y;
         }
@@ -278,7 +284,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #endif
         // a8 store: each compute warp's ring segment -> [excl + warp offset, ...)
 #pragma unroll 1
-        for (int w = 0; w < kComputeWarps; ++w) {
+        for (int w = 0; w < kCW; ++w) {
           const uint32_t c = __shfl_sync(kFull, cnt, w);
           const uint32_t h = __shfl_sync(kFull, hd, w);
           const uint32_t off = __shfl_sync(kFull, incl - cnt, w);
@@ -288,7 +294,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         }
         // release ring space in CTA tile order
         while (ld_volatile_u32(&sm.released) != j) __nanosleep(64);
-        if (lane < kComputeWarps) sm.tail[lane] += cnt;
+        if (lane < kCW) sm.tail[lane] += cnt;
         __syncwarp();
         if (lane == 0) {
           __threadfence_block();
@@ -320,10 +326,10 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #endif
         if (t == kSentinel) break;                    // the writers stop on the ticket ring
         const bool last = (t == a.num_tiles - 1);
-        const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32;   // first element of the warp
-        const float* src = &sm.in[s][w * kBPW * 32];
+        const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kCBPW * 32;   // first element of the warp
+        const float* src = &sm.in[s][w * kCBPW * 32];
         uint32_t cursor = 0;
-        uint32_t fpack[4];
+        uint32_t fpack[kCBPW / 4];
         // Groups of 4 blocks.  The bit transpose packs as many blocks as fit
         // in 32 bits: 4 blocks when every v < 2^8 (F <= 7), 2 when v < 2^16,
         // else 1.  After it, lane q*W + k holds word k of block q (W = 32 /
@@ -333,7 +339,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #ifdef CUSZP_DIAG_NOWORK
         for (int g = 0; g < 0; ++g) {   // diagnostics only: pipeline without the encode work
 #else
-        for (int g = 0; g < kBPW / 4; ++g) {
+        for (int g = 0; g < kCBPW / 4; ++g) {
 #endif
           float x[4];
 #pragma unroll
@@ -441,19 +447,23 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           if constexpr (M == 2) fpack[g] = __byte_perm(fpack[g], 0, 0x4420u);   // blocks (0,1), (2,3)
           if constexpr (M == 4) fpack[g] &= 0xffu;                             // one block
         }
-        // F bytes of the warp's 16 / M blocks (Fig 12 part 1): one store; the
-        // stores also cover the F area's zero padding up to align16(nb)
+        // F bytes of the warp's kCBPW / M blocks (Fig 12 part 1): one store;
+        // the stores also cover the F area's zero padding up to align16(nb)
         // (padding sub-blocks past n encode as zero blocks, F = 0)
-        const uint64_t blk0 = (uint64_t(t) * kTileBlocks + uint64_t(w) * kBPW) / M;
+        const uint64_t blk0 = (uint64_t(t) * kTileBlocks + uint64_t(w) * kCBPW) / M;
         if (lane == 0 && blk0 < align16(a.nb)) {
-          if constexpr (M == 1)
-            *reinterpret_cast<uint4*>(a.out + kHdr + blk0) = make_uint4(fpack[0], fpack[1], fpack[2], fpack[3]);
-          else if constexpr (M == 2)
-            *reinterpret_cast<uint2*>(a.out + kHdr + blk0) =
-                make_uint2(fpack[0] | (fpack[1] << 16), fpack[2] | (fpack[3] << 16));
-          else
-            *reinterpret_cast<uint32_t*>(a.out + kHdr + blk0) =
-                fpack[0] | (fpack[1] << 8) | (fpack[2] << 16) | (fpack[3] << 24);
+          uint32_t fw[4] = {0, 0, 0, 0};                  // the F bytes, little-endian
+#pragma unroll
+          for (int g = 0; g < kCBPW / 4; ++g) {
+            constexpr int kBytes = 4 / M;                   // F bytes per group
+            const int bit = g * kBytes * 8;
+            fw[bit / 32] |= fpack[g] << (bit % 32);
+          }
+          constexpr int kFBytes = kCBPW / M;
+          if constexpr (kFBytes == 16) *reinterpret_cast<uint4*>(a.out + kHdr + blk0) = make_uint4(fw[0], fw[1], fw[2], fw[3]);
+          else if constexpr (kFBytes == 8) *reinterpret_cast<uint2*>(a.out + kHdr + blk0) = make_uint2(fw[0], fw[1]);
+          else if constexpr (kFBytes == 4) *reinterpret_cast<uint32_t*>(a.out + kHdr + blk0) = fw[0];
+          else *reinterpret_cast<uint16_t*>(a.out + kHdr + blk0) = uint16_t(fw[0]);
         }
         __syncwarp();
         if (lane == 0) {
@@ -462,12 +472,12 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           md.cnt[w] = uint16_t(cursor);
           md.head[w] = uint16_t(head & (kRing - 1));
           __threadfence_block();
-          if (atomicAdd(&sm.meta_done[m], 1u) == kComputeWarps - 1) {
+          if (atomicAdd(&sm.meta_done[m], 1u) == kCW - 1) {
             // last warp of the tile: aggregate -> publish at once (look-back, part 1)
             __threadfence_block();
             uint32_t agg = 0;
 #pragma unroll
-            for (int k = 0; k < kComputeWarps; ++k)
+            for (int k = 0; k < kCW; ++k)
               agg += *reinterpret_cast<volatile uint16_t*>(&md.cnt[k]);
             publish_aggregate(a.status, t, agg, epoch);
             trace_put(a.trace, t, 2, global_ns());
