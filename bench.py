@@ -55,6 +55,7 @@ def parse_args():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--config", default="c2_hurricane")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-large", action="store_true", help="skip the 1.12 GB HACC-shaped context measurement")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=10.0)
     return p.parse_args()
@@ -330,6 +331,43 @@ def run_ours(args, rank, world, dev):
     q_bytes = sum(8 * n_of[f] for f, _ in jobs)
     quality["kernel_gbs"] = q_bytes / (sum(q_ms) / 1e3) / 1e9
 
+    # a large field (HACC-shaped, 1.12 GB, REL 1e-3; BASELINE configs[2]) where
+    # launch ramp and drain are amortised: kernel times and roofline fractions
+    # (context for the 100 MB headline fields; inputs >> L2, median of 3)
+    large = None
+    if not args.no_large and world == 1:
+        xl = synth.field_for_config("c3_hacc", device=dev)
+        nl = xl.numel()
+        capl = cz.max_compressed_bytes(nl)
+        wsl = cz.Workspace(nl, dev)
+        outl = torch.empty(capl, dtype=torch.uint8, device=dev)
+        yl = torch.empty(nl, dtype=torch.float32, device=dev)
+        mml = torch.empty(2, dtype=torch.float32, device=dev)
+        tl = {"range": [], "compress": [], "decompress": []}
+        ev4 = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+        for _ in range(4):
+            ev4[0].record(stream)
+            cz.check(lib.cuszp_range(xl.data_ptr(), nl, mml.data_ptr(), wsl.ptr(), wsl.nbytes, sp), "range")
+            ev4[1].record(stream)
+            cz.check(lib.cuszp_compress_minmax(xl.data_ptr(), nl, 1e-3, mml.data_ptr(), 1, outl.data_ptr(), capl,
+                                               out_bytes.data_ptr(), wsl.ptr(), wsl.nbytes, sp), "compress")
+            ev4[2].record(stream)
+            cz.check(lib.cuszp_decompress(outl.data_ptr(), capl, yl.data_ptr(), nl, wsl.ptr(), wsl.nbytes, sp),
+                     "decompress")
+            ev4[3].record(stream)
+            torch.cuda.synchronize(dev)
+            for k, (e0, e1) in zip(tl, ((0, 1), (1, 2), (2, 3))):
+                tl[k].append(ev4[e0].elapsed_time(ev4[e1]) / 1e3)
+        assert cz.last_status(wsl) == cz.OK
+        Sl = int(out_bytes.item())
+        med = {k: float(np.median(v[1:])) for k, v in tl.items()}
+        bl = {"range": 4 * nl, "compress": 4 * nl + Sl, "decompress": Sl + 4 * nl}
+        large = {"workload": "c3_hacc (280,953,867 fp32, 1.12 GB) REL 1e-3", "cr": round(4 * nl / Sl, 3),
+                 **{k: {"us": round(med[k] * 1e6, 1), "algorithmic_gbs": round(bl[k] / med[k] / 1e9, 1),
+                        "frac_of_peak": round(bl[k] / med[k] / 1e9 / peak_hbm()[0], 4)} for k in med}}
+        del xl, yl, outl, wsl
+        torch.cuda.empty_cache()
+
     # block-length variants on the first field at the
     # middle bound: compress and decompress kernels, L2 flushed, median of 5
     f0, rel0 = fields[0], rels[len(rels) // 2]
@@ -412,6 +450,7 @@ def run_ours(args, rank, world, dev):
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
         "gpu_launches": 3 * len(jobs) * K,
         "block_len_variants": {"workload": f"{f0}@{rel0:g}", "unit": "GB/s of fp32 input", **variants},
+        "large_field": large,
         "quality": dict(quality, frac_of_peak=quality["kernel_gbs"] / peak,
                         kernel="cuszp_quality (fused compareData statistics, untimed verification pass)"),
         "clocks": clk,
