@@ -115,7 +115,10 @@ int oracle_compress_minmax_L(const float* x, uint64_t n, float lambda,
  * (means first, then centred sums).  out[0..11] = min, max, range,
  * max_abs_err, max_rel_err, max_pw_rel_err, mse, psnr, nrmse, norm_err,
  * norm_err_norm, pearson; out_counts[0..1] = n, #{|x_i - y_i| > bound}.
- * n must be > 0. */
+ * n must be > 0.  Pinned by the artifact's printed values, closed forms and
+ * numpy's corrcoef -- except norm_err_norm (= ||e||/||x||, reading Q2 of
+ * "parity unpinned" for that one field, the paper prints it
+ * without the data needed to check the normalisation). */
 void oracle_quality(const float* x, const float* y, uint64_t n, double bound,
                     double out[12], uint64_t out_counts[2]);
 
