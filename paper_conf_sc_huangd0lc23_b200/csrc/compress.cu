@@ -353,36 +353,53 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           quantize_fast2(x[2], x[3], two_eb, recip, vmax, resmax, r[2], r[3]);
           // NaN residuals are not caught here (fmax drops NaN) but NaN/Inf data
           // always yield a block with > 25 words below (flagged, R5)
+#ifdef CUSZP_C_EAGER_RARE
           if (__any_sync(kFull, resmax > eb)) {
 #pragma unroll
             for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
           }
-          uint32_t v[4];
-          if constexpr (M == 1) {
+#else
+          // the vote is taken now but acted on after the word counts: the
+          // Lorenzo shuffles and reductions of the (nearly always exact) fast
+          // result do not wait for it; a group that needs R2's correction is
+          // then redone in full
+          const bool rare = __any_sync(kFull, resmax > eb);
+#endif
+          uint32_t v[4], wq[4];
+          auto lorenzo_and_counts = [&]() {
+            if constexpr (M == 1) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
-          } else {
-            // a block continues across its sub-blocks: lane 0 of sub-block q
-            // takes lane 31 of sub-block q-1 unless q starts a block
+              for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
+            } else {
+              // a block continues across its sub-blocks: lane 0 of sub-block q
+              // takes lane 31 of sub-block q-1 unless q starts a block
 #pragma unroll
-            for (int q = 0; q < 4; ++q)
-              v[q] = lorenzo_pack_first(r[q], lane,
-                                        (q % M == 0) ? kRoundMagicBits : __shfl_sync(kFull, r[q > 0 ? q - 1 : 0], 31));
+              for (int q = 0; q < 4; ++q)
+                v[q] = lorenzo_pack_first(r[q], lane,
+                                          (q % M == 0) ? kRoundMagicBits : __shfl_sync(kFull, r[q > 0 ? q - 1 : 0], 31));
+            }
+#ifdef CUSZP_DIAG_TINY
+            v[0] = v[1] = v[2] = v[3] = 0;   // diagnostics only: all zero blocks (wrong output)
+#endif
+            // a5: words per block = bit length of the block's OR of v (= of its max)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              uint32_t b;
+              asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(__reduce_or_sync(kFull, v[q])));   // -1 for 0
+              wq[q] = b + 1;
+            }
+          };
+          lorenzo_and_counts();
+#ifndef CUSZP_C_EAGER_RARE
+          if (rare) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
+            lorenzo_and_counts();
           }
+#endif
           // room in this warp's ring for a worst-case group (4 x 32 words)
           while (head + cursor + 4 * 32 - ld_volatile_u32(&sm.tail[w]) > kRing)
             __nanosleep(CUSZP_C_POLL_NS);
-#ifdef CUSZP_DIAG_TINY
-          v[0] = v[1] = v[2] = v[3] = 0;   // diagnostics only: all zero blocks (wrong output)
-#endif
-          // a5: words per block = bit length of the block's OR of v (= of its max)
-          uint32_t wq[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            uint32_t b;
-            asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(__reduce_or_sync(kFull, v[q])));   // -1 for 0
-            wq[q] = b + 1;
-          }
           if constexpr (M == 2) {                                        // one F per block
             wq[0] = wq[1] = max(wq[0], wq[1]);
             wq[2] = wq[3] = max(wq[2], wq[3]);
