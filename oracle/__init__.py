@@ -81,6 +81,8 @@ def lib():
             h.oracle_compress_L.restype = i32
             h.oracle_compress_minmax_L.argtypes = [vp, u64, f32, vp, i32, i32, vp, u64, vp]
             h.oracle_compress_minmax_L.restype = i32
+            h.oracle_compress_ex.argtypes = [vp, u64, f32, i32, i32, i32, vp, u64, vp]
+            h.oracle_compress_ex.restype = i32
             _lib = h
     return _lib
 
@@ -215,6 +217,17 @@ def compress_L(x, eb: float, mode: int, Lb: int) -> tuple[int, np.ndarray]:
     out = np.zeros(cap, np.uint8)
     nbytes = np.zeros(1, np.uint64)
     st = lib().oracle_compress_L(_ptr(x), x.size, np.float32(eb), int(mode), int(Lb), _ptr(out), cap, _ptr(nbytes))
+    return st, out[: int(nbytes[0])].copy() if st in (OK, ERANGE) else out[:0]
+
+
+def compress_ex(x, eb: float, mode: int, Lb: int = L, order: int = 1) -> tuple[int, np.ndarray]:
+    """Block length Lb and Lorenzo order (1, or 2 = the 2-layer predictor)."""
+    x = _f32(x).ravel()
+    cap = max_compressed_bytes_L(x.size, Lb)
+    out = np.zeros(cap, np.uint8)
+    nbytes = np.zeros(1, np.uint64)
+    st = lib().oracle_compress_ex(_ptr(x), x.size, np.float32(eb), int(mode), int(Lb), int(order), _ptr(out), cap,
+                                  _ptr(nbytes))
     return st, out[: int(nbytes[0])].copy() if st in (OK, ERANGE) else out[:0]
 
 

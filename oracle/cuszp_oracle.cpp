@@ -20,6 +20,9 @@
 #include <cstring>
 #include <vector>
 
+int prequantize_guarded(const float* x, size_t n, float eb_abs, int32_t* q, float guard);
+void block_lorenzo_order(const int32_t* q, size_t nb, int L, int order, int32_t* l);
+
 namespace {
 
 const int L = 32;                     /* default block length, R1 */
@@ -29,6 +32,7 @@ bool valid_block_len(int Lb) { return Lb == 8 || Lb == 16 || Lb == 32 || Lb == 6
 int log2_of(int Lb) { int k = 0; while ((1 << k) < Lb) ++k; return k; }
 const int HEADER_BYTES = 32;          /* R10 */
 const float GUARD = 4194304.0f;       /* 2^22, R5 */
+const float GUARD2 = 2097152.0f;      /* 2^21: 2-layer Lorenzo keeps |l| <= 2^23 (R17) */
 const int MAX_F = 24;                 /* consequence of the guard, R5 */
 
 uint64_t align16(uint64_t v) { return (v + 15u) & ~uint64_t(15); }
@@ -65,7 +69,8 @@ void write_header(uint8_t* out, uint64_t n, int mode, int status, float eb_abs,
  * Fig 2): Quantisation and Prediction -> Fixed-length Encoding ->
  * Global Synchronization -> Block Bit-shuffle. */
 int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int mode,
-                     uint8_t* out, uint64_t cap, uint64_t* out_bytes, int L) {
+                     uint8_t* out, uint64_t cap, uint64_t* out_bytes, int L, int order = 1) {
+  mode |= (order == 2) ? 0x10 : 0;                      /* header: predictor order (R17) */
   const uint64_t nb = (n + L - 1) / L;                  /* number of blocks N */
   if (cap < oracle_max_compressed_bytes_L(n, L)) return ORACLE_ENOSPACE;
   std::memset(out, 0, size_t(HEADER_BYTES + align16(nb)));
@@ -83,7 +88,7 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
 
   /* (1) Pre-quantisation, the only lossy step. */
   std::vector<int32_t> r(static_cast<size_t>(nb * L), 0);            /* zero pad, R8 */
-  if (oracle_prequantize(x, size_t(n), eb_abs, r.data()) != ORACLE_OK) {
+  if (prequantize_guarded(x, size_t(n), eb_abs, r.data(), order == 2 ? GUARD2 : GUARD) != ORACLE_OK) {
     write_header(out, n, mode, ORACLE_ERANGE, eb_abs, eb_in, 0, L);
     *out_bytes = HEADER_BYTES + align16(nb);
     return ORACLE_ERANGE;
@@ -91,7 +96,7 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
 
   /* (1') Lorenzo prediction inside each block. */
   std::vector<int32_t> l(static_cast<size_t>(nb * L));
-  oracle_block_lorenzo_L(r.data(), size_t(nb), L, l.data());
+  block_lorenzo_order(r.data(), size_t(nb), L, order, l.data());
 
   /* (2) Fixed-length encoding: F_k and CmpL_k per block,
    *     giving the BlockOffsetArray. */
@@ -142,6 +147,13 @@ void oracle_value_range(const float* x, size_t n, float* mn, float* mx) {
 }
 
 int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q) {
+  return prequantize_guarded(x, n, eb_abs, q, GUARD);
+}
+
+}  // extern "C"
+
+/* R2 with the guard of the predictor order (R5 / R17). */
+int prequantize_guarded(const float* x, size_t n, float eb_abs, int32_t* q, float guard) {
   /* r_i = round(d_i / 2eb), guaranteeing |r_i * 2eb - d_i| <= eb.
    * fp32 op sequence R2 (shared by definition, not by code, with the GPU):
    *   two_eb = eb + eb; recip = 1 / two_eb           (fp32, once)
@@ -156,7 +168,7 @@ int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q) {
   for (size_t i = 0; i < n; ++i) {
     const double p = double(x[i]) * double(recip);      /* exact */
     const double r0d = std::nearbyint(p);
-    if (!(std::fabs(r0d) < double(GUARD))) return ORACLE_ERANGE;
+    if (!(std::fabs(r0d) < double(guard))) return ORACLE_ERANGE;
     const float r0 = float(r0d);                         /* exact, |r0| < 2^22 */
     const float res = std::fmaf(-r0, two_eb, x[i]);
     int32_t r = int32_t(r0);
@@ -166,6 +178,23 @@ int oracle_prequantize(const float* x, size_t n, float eb_abs, int32_t* q) {
   }
   return ORACLE_OK;
 }
+
+/* 2-layer 1D Lorenzo inside each block (R17):
+ * l_i = r_i - 2 r_{i-1} + r_{i-2}, r_{-1} = r_{-2} = 0 at every block start. */
+void block_lorenzo_order(const int32_t* q, size_t nb, int L, int order, int32_t* l) {
+  if (order != 2) { oracle_block_lorenzo_L(q, nb, L, l); return; }
+  for (size_t k = 0; k < nb; ++k) {
+    const int32_t* r = q + k * L;
+    int32_t* lk = l + k * L;
+    for (int i = 0; i < L; ++i) {
+      const int32_t p1 = (i >= 1) ? r[i - 1] : 0;
+      const int32_t p2 = (i >= 2) ? r[i - 2] : 0;
+      lk[i] = r[i] - 2 * p1 + p2;
+    }
+  }
+}
+
+extern "C" {
 
 void oracle_block_lorenzo(const int32_t* q, size_t nb, int32_t* l) {
   oracle_block_lorenzo_L(q, nb, L, l);
@@ -264,20 +293,26 @@ int oracle_compress(const float* x, uint64_t n, float eb, int mode,
 
 int oracle_compress_L(const float* x, uint64_t n, float eb, int mode, int L,
                       uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
-  if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr || !valid_block_len(L))
+  return oracle_compress_ex(x, n, eb, mode, L, 1, out, cap, out_bytes);
+}
+
+int oracle_compress_ex(const float* x, uint64_t n, float eb, int mode, int L, int order,
+                       uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  if ((n > 0 && x == nullptr) || out == nullptr || out_bytes == nullptr || !valid_block_len(L) ||
+      (order != 1 && order != 2))
     return ORACLE_EINVAL;
   if (mode == 0) {                                      /* ABS: eb = delta */
     if (!eb_usable(eb)) return ORACLE_EINVAL;
-    return compress_with_eb(x, n, eb, eb, 0, out, cap, out_bytes, L);
+    return compress_with_eb(x, n, eb, eb, 0, out, cap, out_bytes, L, order);
   }
   if (mode == 1) {                                      /* REL: eb = lambda * r */
     if (!(eb > 0.0f) || !std::isfinite(eb)) return ORACLE_EINVAL;
-    if (n == 0) return compress_with_eb(x, 0, 0.0f, eb, 1, out, cap, out_bytes, L);
+    if (n == 0) return compress_with_eb(x, 0, 0.0f, eb, 1, out, cap, out_bytes, L, order);
     float mn, mx;
     oracle_value_range(x, size_t(n), &mn, &mx);
     const float range = mx - mn;                        /* R3: fp32 */
     const float eb_abs = eb * range;
-    return compress_with_eb(x, n, eb_abs, eb, 1, out, cap, out_bytes, L);
+    return compress_with_eb(x, n, eb_abs, eb, 1, out, cap, out_bytes, L, order);
   }
   return ORACLE_EINVAL;
 }
@@ -313,6 +348,7 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
   if (!(in[0] == 'C' && in[1] == 'S' && in[2] == 'Z' && in[3] == 'P') ||
       in[4] != 1 || in[7] < 3 || in[7] > 7) return ORACLE_ECORRUPT;
   const int L = 1 << in[7];                             /* block length from the header */
+  const int order = (in[5] & 0x10) ? 2 : 1;             /* predictor order from the header (R17) */
   if (in[6] != ORACLE_OK) return in[6] == ORACLE_ERANGE ? ORACLE_ERANGE : ORACLE_ECORRUPT;
   if (get_u64(in + 8) != n) return ORACLE_EINVAL;
   if (n == 0) return ORACLE_OK;
@@ -338,10 +374,17 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
   for (uint64_t k = 0; k < nb; ++k) {
     int32_t l[MAX_L];
     oracle_decode_block_L(in + p0 + sync_offset[k], fixed_length[k], L, l);
-    /* reverse Lorenzo: r_i = r_{i-1} + l_i inside the block */
-    int32_t r = 0;
+    /* reverse Lorenzo: r_i = r_{i-1} + l_i inside the block (order 2:
+     * r_i = l_i + 2 r_{i-1} - r_{i-2}) */
+    int32_t r = 0, r1 = 0, r2 = 0;
     for (int i = 0; i < L; ++i) {
-      r += l[i];
+      if (order == 2) {
+        r = l[i] + 2 * r1 - r2;
+        r2 = r1;
+        r1 = r;
+      } else {
+        r += l[i];
+      }
       const uint64_t idx = k * L + uint64_t(i);
       /* d'_i = r_i * 2eb */
       if (idx < n) out[idx] = float(r) * two_eb;

@@ -109,6 +109,13 @@ int oracle_compress_minmax_L(const float* x, uint64_t n, float lambda,
                              const float* minmax, int n_pairs, int L,
                              uint8_t* out, uint64_t cap, uint64_t* out_bytes);
 
+/* ---- 2-layer Lorenzo (DESIGN R17) --
+ * order 2: l_i = r_i - 2 r_{i-1} + r_{i-2} inside each block (r_{-1} =
+ * r_{-2} = 0), guard |r0| < 2^21 so F <= 24; header mode byte bit 4 (0x10)
+ * marks it and oracle_decompress inverts it.  order 1 = oracle_compress_L. */
+int oracle_compress_ex(const float* x, uint64_t n, float eb, int mode, int L, int order,
+                       uint8_t* out, uint64_t cap, uint64_t* out_bytes);
+
 /* ---- reconstruction quality -------------------
  * The statistics of the paper's artifact output (QCAT compareData,
  * P:1918-1933) and PSNR (sec 2.1), in fp64, two plain passes

@@ -35,14 +35,20 @@ def decode_to_ints(buf: bytes) -> tuple[dict, list[int], list[int]]:
         nbytes = (f + 1) * Lb // 8
         blk = buf[pos:pos + nbytes]
         pos += nbytes
-        r = 0
+        r, r1, r2 = 0, 0, 0
+        order2 = bool(h["mode"] & 0x10)          # 2-layer Lorenzo (DESIGN R17)
         for j in range(Lb):
             neg = (blk[j // 8] >> (j % 8)) & 1
             mag = 0
             for p in range(f):
                 byte = blk[(p + 1) * (Lb // 8) + j // 8]
                 mag |= ((byte >> (j % 8)) & 1) << p
-            r += -mag if neg else mag
+            l = -mag if neg else mag
+            if order2:
+                r = l + 2 * r1 - r2
+                r2, r1 = r1, r
+            else:
+                r += l
             r_all.append(r)
     h["consumed"] = pos
     return h, F, r_all
