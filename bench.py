@@ -374,30 +374,34 @@ def run_ours(args, rank, world, dev):
     x0, n0 = xs[f0], n_of[f0]
     cz.check(lib.cuszp_range(x0.data_ptr(), n0, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
     variants = {}
-    for Lb in (32, 64, 128):
+    for Lb, order in ((32, 1), (64, 1), (128, 1), (32, 2)):
         tc, td = [], []
         capL = cz.max_compressed_bytes(n0, Lb)
         outL = out if capL <= cap else torch.empty(capL, dtype=torch.uint8, device=dev)
         for _ in range(6):
             flush_l2()
             qev[0].record(stream)
-            cz.check(lib.cuszp_compress_minmax_L(x0.data_ptr(), n0, float(rel0), mm_local.data_ptr(), 1, Lb,
-                                                 outL.data_ptr(), capL, out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
-                                                 sp), "compress_L")
+            if order == 1:
+                cz.check(lib.cuszp_compress_minmax_L(x0.data_ptr(), n0, float(rel0), mm_local.data_ptr(), 1, Lb,
+                                                     outL.data_ptr(), capL, out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
+                                                     sp), "compress_L")
+            else:   # 2-layer Lorenzo: REL through the range kernel too
+                cz.check(lib.cuszp_compress_ex(x0.data_ptr(), n0, float(rel0), cz.REL, Lb, order, outL.data_ptr(),
+                                               capL, out_bytes.data_ptr(), ws.ptr(), ws.nbytes, sp), "compress_ex")
             qev[1].record(stream)
             torch.cuda.synchronize(dev)
             tc.append(qev[0].elapsed_time(qev[1]))
             flush_l2()
             qev[0].record(stream)
-            cz.check(lib.cuszp_decompress_L(outL.data_ptr(), capL, y.data_ptr(), n0, Lb, ws.ptr(), ws.nbytes, sp),
-                     "decompress_L")
+            cz.check(lib.cuszp_decompress_ex(outL.data_ptr(), capL, y.data_ptr(), n0, Lb, order, ws.ptr(),
+                                             ws.nbytes, sp), "decompress_ex")
             qev[1].record(stream)
             torch.cuda.synchronize(dev)
             td.append(qev[0].elapsed_time(qev[1]))
         assert cz.last_status(ws) == cz.OK
         SL = int(out_bytes.item())
         tcm, tdm = float(np.median(tc[1:])) / 1e3, float(np.median(td[1:])) / 1e3
-        variants[str(Lb)] = {"cr": round(4 * n0 / SL, 3),
+        variants[str(Lb) if order == 1 else f"{Lb}_lorenzo2"] = {"cr": round(4 * n0 / SL, 3),
                              "compress_kernel_gbs": round(4 * n0 / tcm / 1e9, 1),
                              "decompress_kernel_gbs": round(4 * n0 / tdm / 1e9, 1),
                              "compress_frac_of_peak": round((4 * n0 + SL) / tcm / 1e9 / peak_hbm()[0], 4),

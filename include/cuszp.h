@@ -140,6 +140,19 @@ int cuszp_compress_minmax_L(const float* d_in, size_t n, float lambda,
 int cuszp_decompress_L(const void* d_in, size_t in_bytes, float* d_out, size_t n, int block_len,
                        void* d_ws, size_t ws_bytes, void* stream);
 
+/* ---- 2-layer Lorenzo predictor ----
+ * order 1: the paper's 1D 1-layer predictor (the calls above); order 2:
+ * l_i = r_i - 2 r_{i-1} + r_{i-2} inside each block (r_{-1} = r_{-2} = 0),
+ * R5 guard |r0| < 2^21 (so F <= 24), header mode byte bit 4 (0x10) set;
+ * block_len must be 32 for order 2.  Decompression must be given the
+ * stream's order (another order in the header: async ECORRUPT).  Sizes and
+ * errors as for the _L calls; order outside {1, 2}: EINVAL. */
+int cuszp_compress_ex(const float* d_in, size_t n, float eb, int mode, int block_len, int order,
+                      void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
+                      void* d_ws, size_t ws_bytes, void* stream);
+int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t n, int block_len,
+                        int order, void* d_ws, size_t ws_bytes, void* stream);
+
 /* Status of the last compress/decompress call made with this workspace.
  * SYNCHRONISES `stream`.  Returns a cuszp_status (or ECUDA). */
 int cuszp_last_status(const void* d_ws, void* stream);

@@ -114,7 +114,7 @@ def value_range(x: torch.Tensor, ws: Workspace | None = None, out: torch.Tensor 
 
 def compress(x: torch.Tensor, eb: float, mode="rel", out: torch.Tensor | None = None,
              out_bytes: torch.Tensor | None = None, ws: Workspace | None = None, stream=None,
-             block_len: int = BLOCK_LEN):
+             block_len: int = BLOCK_LEN, order: int = 1):
     """Compress a float32 CUDA tensor.  Returns (stream buffer uint8 tensor of
     capacity max_compressed_bytes(n), device int64 tensor [1] holding the
     exact stream length).  Asynchronous; data errors land in the header."""
@@ -127,9 +127,9 @@ def compress(x: torch.Tensor, eb: float, mode="rel", out: torch.Tensor | None = 
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
     ws = _workspace(n, x.device, ws)
-    check(lib().cuszp_compress_L(x.data_ptr(), n, float(eb), _mode(mode), int(block_len), out.data_ptr(),
-                                 out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
-          "cuszp_compress")
+    check(lib().cuszp_compress_ex(x.data_ptr(), n, float(eb), _mode(mode), int(block_len), int(order),
+                                  out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
+                                  _stream_ptr(stream)), "cuszp_compress")
     return out, out_bytes
 
 
@@ -152,7 +152,7 @@ def compress_minmax(x: torch.Tensor, lam: float, minmax: torch.Tensor, out: torc
 
 
 def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None, in_bytes: int | None = None,
-               ws: Workspace | None = None, stream=None, block_len: int = BLOCK_LEN) -> torch.Tensor:
+               ws: Workspace | None = None, stream=None, block_len: int = BLOCK_LEN, order: int = 1) -> torch.Tensor:
     """Decompress a device stream into n float32 values (asynchronous)."""
     _require_cuda(stream_buf, "stream_buf", torch.uint8)
     if out is None:
@@ -160,8 +160,8 @@ def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None
     _require_cuda(out, "out", torch.float32)
     ws = _workspace(n, stream_buf.device, ws)
     nbytes = stream_buf.numel() if in_bytes is None else int(in_bytes)
-    check(lib().cuszp_decompress_L(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), int(block_len), ws.ptr(),
-                                   ws.nbytes, _stream_ptr(stream)), "cuszp_decompress")
+    check(lib().cuszp_decompress_ex(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), int(block_len),
+                                    int(order), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_decompress")
     return out
 
 

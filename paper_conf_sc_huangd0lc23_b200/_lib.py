@@ -25,6 +25,7 @@ SYMBOLS = (
     "cuszp_status_string", "cuszp_version", "cuszp_quality_workspace_bytes", "cuszp_quality",
     "cuszp_compress_host_async", "cuszp_decompress_host_async",
     "cuszp_compress_L", "cuszp_compress_minmax_L", "cuszp_decompress_L", "cuszp_max_compressed_bytes_L",
+    "cuszp_compress_ex", "cuszp_decompress_ex",
 )
 
 _lock = threading.Lock()
@@ -71,6 +72,10 @@ def _declare(h):
     h.cuszp_compress_host_async.restype = i32
     h.cuszp_decompress_host_async.argtypes = [vp, sz, vp, sz, vp, vp, vp, sz, vp]
     h.cuszp_decompress_host_async.restype = i32
+    h.cuszp_compress_ex.argtypes = [vp, sz, f32, i32, i32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_compress_ex.restype = i32
+    h.cuszp_decompress_ex.argtypes = [vp, sz, vp, sz, i32, i32, vp, sz, vp]
+    h.cuszp_decompress_ex.restype = i32
     h.cuszp_max_compressed_bytes_L.argtypes = [sz, i32]
     h.cuszp_max_compressed_bytes_L.restype = sz
     h.cuszp_compress_L.argtypes = [vp, sz, f32, i32, i32, vp, sz, vp, vp, sz, vp]

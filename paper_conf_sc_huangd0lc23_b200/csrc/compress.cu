@@ -161,8 +161,22 @@ __device__ __forceinline__ uint32_t pack4(uint32_t a, uint32_t b, uint32_t c, ui
 // sub-blocks sharing one F; word k of sub-block i of a block sits at
 // M k + i of the block's payload (a plane is L/8 bytes, element j at byte
 // j/8, bit j%8 -- R9 generalised).  M = 1 is the paper's default L = 32.
-template <int M>
+// lane j holds the biased r_j of one block -> v_j for the 2-layer Lorenzo
+// (R17): l_j = r_j - 2 r_{j-1} + r_{j-2}, r_{-1} = r_{-2} = 0
+__device__ __forceinline__ uint32_t lorenzo2_pack(uint32_t rb, int lane) {
+  uint32_t p1 = __shfl_up_sync(kFull, rb, 1), p2 = __shfl_up_sync(kFull, rb, 2);
+  p1 = lane >= 1 ? p1 : kRoundMagicBits;
+  p2 = lane >= 2 ? p2 : kRoundMagicBits;
+  const int l = int(rb - p1) - int(p1 - p2);                 // the biases cancel
+  const uint32_t a = uint32_t(l < 0 ? -l : l);
+  return (a << 1) | (uint32_t(l) >> 31);
+}
+
+// O = Lorenzo order: 1 (the paper's 1D 1-layer predictor) or 2 (2-layer,
+// SURVEY 8(f) rank 4; L = 32 only).
+template <int M, int O>
 __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(CompressArgs a) {
+  static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
   extern __shared__ __align__(128) unsigned char smem_raw[];
   CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
@@ -369,7 +383,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           auto lorenzo_and_counts = [&]() {
             if constexpr (M == 1) {
 #pragma unroll
-              for (int q = 0; q < 4; ++q) v[q] = lorenzo_pack(r[q], lane);
+              for (int q = 0; q < 4; ++q) v[q] = (O == 2) ? lorenzo2_pack(r[q], lane) : lorenzo_pack(r[q], lane);
             } else {
               // a block continues across its sub-blocks: lane 0 of sub-block q
               // takes lane 31 of sub-block q-1 unless q starts a block
@@ -512,7 +526,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   // R5 guard: some |r0| >= 2^22 (NaN and Inf included)
   uint32_t flag = 0;
   if (!eb_ok) flag = (a.n > 0) ? kBadRange : 0u;
-  else if (!(vmax < kGuard) || wmax > uint32_t(kMaxBlockWords)) flag = kBadRange;
+  else if (!(vmax < (O == 2 ? 0.5f * kGuard : kGuard)) || wmax > uint32_t(kMaxBlockWords)) flag = kBadRange;   // R5 / R17
 
   if (cta_finish(a.ws, flag)) {
     uint32_t final_status = CUSZP_OK;
@@ -526,7 +540,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       uint8_t* h = a.out;                                   // header (R10)
       *reinterpret_cast<uint32_t*>(h) = 0x505A5343u;        // "CSZP"
       h[4] = CUSZP_VERSION;
-      h[5] = uint8_t(a.mode);
+      h[5] = uint8_t(a.mode | (O == 2 ? 0x10 : 0));        // predictor order (R17)
       h[6] = uint8_t(final_status);
       h[7] = uint8_t(5 + (M == 2 ? 1 : M == 4 ? 2 : 0));   // log2(L)
       *reinterpret_cast<uint64_t*>(h + 8) = a.n;
@@ -542,20 +556,22 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 }
 
 namespace {
-template <int M>
+template <int M, int O = 1>
 cudaError_t configure_m(int* occ) {
   const int smem = int(sizeof(CompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M>, kCThreads, smem);
+  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M, O>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M, O>, kCThreads, smem);
   return e;
 }
 }  // namespace
 
 cudaError_t compress_configure(int M, int* occ) {
+  int occ2 = 0;
+  if (M == 1 && configure_m<1, 2>(&occ2) != cudaSuccess) return cudaErrorUnknown;
   return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
 }
 
-cudaError_t compress_launch(int M, unsigned grid, const CompressArgs& a, cudaStream_t s) {
+cudaError_t compress_launch(int M, int order, unsigned grid, const CompressArgs& a, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kCThreads);
@@ -566,9 +582,10 @@ cudaError_t compress_launch(int M, unsigned grid, const CompressArgs& a, cudaStr
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (M == 1) return cudaLaunchKernelEx(&cfg, compress_kernel<1>, a);
-  if (M == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<2>, a);
-  return cudaLaunchKernelEx(&cfg, compress_kernel<4>, a);
+  if (order == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 2>, a);
+  if (M == 1) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1>, a);
+  if (M == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<2, 1>, a);
+  return cudaLaunchKernelEx(&cfg, compress_kernel<4, 1>, a);
 }
 
 size_t compress_smem_bytes() { return sizeof(CompressSmem); }

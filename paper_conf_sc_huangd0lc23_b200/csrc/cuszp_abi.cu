@@ -69,9 +69,9 @@ uint32_t status_capacity(size_t ws_bytes) {
 
 int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const float* d_minmax,
                     int n_pairs, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
-                    void* d_ws, size_t ws_bytes, cudaStream_t stream, int L = kL) {
+                    void* d_ws, size_t ws_bytes, cudaStream_t stream, int L = kL, int order = 1) {
   const int M = sub_blocks(L);
-  if (M == 0) return CUSZP_EINVAL;
+  if (M == 0 || (order != 1 && order != 2) || (order == 2 && M != 1)) return CUSZP_EINVAL;
   if (out_capacity < cuszp_max_compressed_bytes_L(n, L) || ws_bytes < cuszp_workspace_bytes(n))
     return CUSZP_ENOSPACE;
   DeviceInfo di;
@@ -95,7 +95,7 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  return compress_launch(M, unsigned(grid), a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+  return compress_launch(M, order, unsigned(grid), a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
 }  // namespace
@@ -170,7 +170,15 @@ int cuszp_compress(const float* d_in, size_t n, float eb, int mode, void* d_out,
 int cuszp_compress_L(const float* d_in, size_t n, float eb, int mode, int block_len, void* d_out,
                      size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes,
                      void* stream) {
-  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || sub_blocks(block_len) == 0)
+  return cuszp_compress_ex(d_in, n, eb, mode, block_len, 1, d_out, out_capacity, d_out_bytes, d_ws, ws_bytes,
+                           stream);
+}
+
+int cuszp_compress_ex(const float* d_in, size_t n, float eb, int mode, int block_len, int order, void* d_out,
+                      size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes,
+                      void* stream) {
+  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || sub_blocks(block_len) == 0 ||
+      (order != 1 && order != 2) || (order == 2 && block_len != kL))
     return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
@@ -179,7 +187,7 @@ int cuszp_compress_L(const float* d_in, size_t n, float eb, int mode, int block_
   if (mode == CUSZP_ABS) {
     if (!eb_is_normal(eb)) return CUSZP_EINVAL;
     return launch_compress(d_in, n, CUSZP_ABS, eb, nullptr, 0, d_out, out_capacity, d_out_bytes, d_ws,
-                           ws_bytes, s, block_len);
+                           ws_bytes, s, block_len, order);
   }
   if (mode == CUSZP_REL) {
     if (!(eb > 0.0f) || !(eb - eb == 0.0f)) return CUSZP_EINVAL;
@@ -191,7 +199,7 @@ int cuszp_compress_L(const float* d_in, size_t n, float eb, int mode, int block_
       if (st != CUSZP_OK) return st;
     }
     return launch_compress(d_in, n, CUSZP_REL, eb, n > 0 ? ws->minmax : nullptr, n > 0 ? 1 : 0, d_out,
-                           out_capacity, d_out_bytes, d_ws, ws_bytes, s, block_len);
+                           out_capacity, d_out_bytes, d_ws, ws_bytes, s, block_len, order);
   }
   return CUSZP_EINVAL;
 }
@@ -224,8 +232,15 @@ int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n, 
 
 int cuszp_decompress_L(const void* d_in, size_t in_bytes, float* d_out, size_t n, int block_len, void* d_ws,
                        size_t ws_bytes, void* stream) {
+  return cuszp_decompress_ex(d_in, in_bytes, d_out, n, block_len, 1, d_ws, ws_bytes, stream);
+}
+
+int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t n, int block_len, int order,
+                        void* d_ws, size_t ws_bytes, void* stream) {
   const int M = sub_blocks(block_len);
-  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr || M == 0) return CUSZP_EINVAL;
+  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr || M == 0 ||
+      (order != 1 && order != 2) || (order == 2 && M != 1))
+    return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
     return CUSZP_EINVAL;
@@ -248,7 +263,7 @@ int cuszp_decompress_L(const void* d_in, size_t in_bytes, float* d_out, size_t n
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  return decompress_launch(M, unsigned(grid), a, s) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+  return decompress_launch(M, order, unsigned(grid), a, s) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
 int cuszp_last_status(const void* d_ws, void* stream) {

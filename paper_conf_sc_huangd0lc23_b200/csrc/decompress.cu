@@ -73,9 +73,10 @@ static_assert(kBarFree0 + 2 <= 16, "named barriers");
 // M = L / 32: see compress.cu -- sub-block i of a block
 // finds its word k at M k + i of the block's payload, and the in-block
 // prefix sum (a11) runs over the block's M sub-blocks.
-template <int M>
+template <int M, int O>
 __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kernel(DecompressArgs a) {
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
+  static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
   constexpr uint32_t kLog2L = 5 + (M == 2 ? 1 : M == 4 ? 2 : 0);
   extern __shared__ __align__(128) unsigned char smem_raw[];
   DecompressSmem& sm = *reinterpret_cast<DecompressSmem*>(smem_raw);
@@ -97,7 +98,9 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     const uint64_t hn = *reinterpret_cast<const uint64_t*>(h + 8);
     eb = *reinterpret_cast<const float*>(h + 16);
     const uint64_t pbytes = *reinterpret_cast<const uint64_t*>(h + 24);
-    if (magic != 0x505A5343u || h[4] != CUSZP_VERSION || h[7] != kLog2L) err = CUSZP_ECORRUPT;
+    if (magic != 0x505A5343u || h[4] != CUSZP_VERSION || h[7] != kLog2L ||
+        ((h[5] & 0x10) != 0) != (O == 2))                   // predictor order (R17)
+      err = CUSZP_ECORRUPT;
     else if (h[6] != CUSZP_OK) err = (h[6] == CUSZP_ERANGE) ? CUSZP_ERANGE : CUSZP_ECORRUPT;
     else if (hn != a.n) err = CUSZP_EINVAL;
     else if (a.n > 0) {
@@ -373,12 +376,32 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           if constexpr (M >= 2) incl = scan_step_up(incl, 8, kSeg);
           if constexpr (M >= 4) incl = scan_step_up(incl, 16, kSeg);
           const int carry = incl - e3;
+          e0 += carry;
+          e1 += carry;
+          e2 += carry;
+          e3 = incl;
+          if constexpr (O == 2) {
+            // 2-layer Lorenzo (R17): the first prefix sum gave r_j - r_{j-1};
+            // a second one over the block gives r_j
+            e1 += e0;
+            e2 += e1;
+            e3 += e2;
+            int inc2 = e3;
+            inc2 = scan_step_up(inc2, 1, kSeg);
+            inc2 = scan_step_up(inc2, 2, kSeg);
+            inc2 = scan_step_up(inc2, 4, kSeg);
+            const int c2 = inc2 - e3;
+            e0 += c2;
+            e1 += c2;
+            e2 += c2;
+            e3 = inc2;
+          }
           // a12: d' = r * 2eb
           float4 d;
-          d.x = __fmul_rn(__int2float_rn(e0 + carry), two_eb);
-          d.y = __fmul_rn(__int2float_rn(e1 + carry), two_eb);
-          d.z = __fmul_rn(__int2float_rn(e2 + carry), two_eb);
-          d.w = __fmul_rn(__int2float_rn(incl), two_eb);
+          d.x = __fmul_rn(__int2float_rn(e0), two_eb);
+          d.y = __fmul_rn(__int2float_rn(e1), two_eb);
+          d.z = __fmul_rn(__int2float_rn(e2), two_eb);
+          d.w = __fmul_rn(__int2float_rn(e3), two_eb);
           float* o = outp + g * 128;
           if (!last) {
             *reinterpret_cast<float4*>(o) = d;
@@ -413,20 +436,22 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 }
 
 namespace {
-template <int M>
+template <int M, int O = 1>
 cudaError_t configure_m(int* occ) {
   const int smem = int(sizeof(DecompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M>, kDThreads, smem);
+  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O>, kDThreads, smem);
   return e;
 }
 }  // namespace
 
 cudaError_t decompress_configure(int M, int* occ) {
+  int occ2 = 0;
+  if (M == 1 && configure_m<1, 2>(&occ2) != cudaSuccess) return cudaErrorUnknown;
   return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
 }
 
-cudaError_t decompress_launch(int M, unsigned grid, const DecompressArgs& a, cudaStream_t s) {
+cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kDThreads);
@@ -437,9 +462,10 @@ cudaError_t decompress_launch(int M, unsigned grid, const DecompressArgs& a, cud
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (M == 1) return cudaLaunchKernelEx(&cfg, decompress_kernel<1>, a);
-  if (M == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<2>, a);
-  return cudaLaunchKernelEx(&cfg, decompress_kernel<4>, a);
+  if (order == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 2>, a);
+  if (M == 1) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1>, a);
+  if (M == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<2, 1>, a);
+  return cudaLaunchKernelEx(&cfg, decompress_kernel<4, 1>, a);
 }
 
 size_t decompress_smem_bytes() { return sizeof(DecompressSmem); }

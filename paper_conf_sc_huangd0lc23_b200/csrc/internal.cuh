@@ -431,9 +431,9 @@ constexpr int kQualityMaxGrid = 2048;
 // Kernels templated on M = L / 32 are launched through these host wrappers
 // defined next to them (compress.cu / decompress.cu): M in {1, 2, 4}.
 cudaError_t compress_configure(int M, int* occupancy);        // smem attribute + CTAs per SM
-cudaError_t compress_launch(int M, unsigned grid, const CompressArgs& a, cudaStream_t s);
+cudaError_t compress_launch(int M, int order, unsigned grid, const CompressArgs& a, cudaStream_t s);
 cudaError_t decompress_configure(int M, int* occupancy);
-cudaError_t decompress_launch(int M, unsigned grid, const DecompressArgs& a, cudaStream_t s);
+cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s);
 __global__ void quality_kernel(QualityArgs a);
 __global__ void range_kernel(RangeArgs a);
 int launch_copy_len(void* dst, const void* src, const unsigned long long* d_len, uint64_t cap,
