@@ -88,23 +88,28 @@ class Workspace:
 _ws_cache: dict = {}
 
 
-def _workspace(n: int, device, ws: Workspace | None) -> Workspace:
+def _workspace(n: int, device, ws: Workspace | None, stream=None) -> Workspace:
+    """The caller's workspace, or a cached one per (device, stream the call
+    is launched on): calls on different streams never share a workspace."""
     if ws is not None:
         if not ws.fits(n):
             raise CuszpError(ENOSPACE, "workspace too small")
         return ws
-    key = (device.index if device.index is not None else torch.cuda.current_device(), torch.cuda.current_stream(device).cuda_stream)
+    dev_index = device.index if device.index is not None else torch.cuda.current_device()
+    s = stream if stream is not None else torch.cuda.current_stream(torch.device("cuda", dev_index))
+    key = (dev_index, int(s.cuda_stream))
     w = _ws_cache.get(key)
     if w is None or not w.fits(n):
         w = Workspace(max(int(n), 1 << 20), device)
         _ws_cache[key] = w
+        s.wait_stream(torch.cuda.current_stream(torch.device("cuda", dev_index)))   # zeroed before first use
     return w
 
 
 def value_range(x: torch.Tensor, ws: Workspace | None = None, out: torch.Tensor | None = None, stream=None):
     """(min, max) of x on the device as a float32 tensor of 2 (Eq 1's r)."""
     _require_cuda(x, "x", torch.float32)
-    ws = _workspace(x.numel(), x.device, ws)
+    ws = _workspace(x.numel(), x.device, ws, stream)
     if out is None:
         out = torch.empty(2, dtype=torch.float32, device=x.device)
     check(lib().cuszp_range(x.data_ptr(), x.numel(), out.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
@@ -126,7 +131,7 @@ def compress(x: torch.Tensor, eb: float, mode="rel", out: torch.Tensor | None = 
     _require_cuda(out, "out", torch.uint8)
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
-    ws = _workspace(n, x.device, ws)
+    ws = _workspace(n, x.device, ws, stream)
     check(lib().cuszp_compress_ex(x.data_ptr(), n, float(eb), _mode(mode), int(block_len), int(order),
                                   out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
                                   _stream_ptr(stream)), "cuszp_compress")
@@ -144,7 +149,7 @@ def compress_minmax(x: torch.Tensor, lam: float, minmax: torch.Tensor, out: torc
         out = torch.empty(max_compressed_bytes(n, block_len), dtype=torch.uint8, device=x.device)
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
-    ws = _workspace(n, x.device, ws)
+    ws = _workspace(n, x.device, ws, stream)
     check(lib().cuszp_compress_minmax_L(x.data_ptr(), n, float(lam), minmax.data_ptr(), minmax.numel() // 2,
                                         int(block_len), out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(),
                                         ws.nbytes, _stream_ptr(stream)), "cuszp_compress_minmax")
@@ -158,7 +163,7 @@ def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None
     if out is None:
         out = torch.empty(int(n), dtype=torch.float32, device=stream_buf.device)
     _require_cuda(out, "out", torch.float32)
-    ws = _workspace(n, stream_buf.device, ws)
+    ws = _workspace(n, stream_buf.device, ws, stream)
     nbytes = stream_buf.numel() if in_bytes is None else int(in_bytes)
     check(lib().cuszp_decompress_ex(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), int(block_len),
                                     int(order), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_decompress")
@@ -169,7 +174,7 @@ def last_status(ws: Workspace | None = None, device=None, stream=None) -> int:
     """Status of the last call on ``ws`` (synchronises the stream)."""
     if ws is None:
         device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
-        ws = _workspace(1, device, None)
+        ws = _workspace(1, device, None, stream)
     return int(lib().cuszp_last_status(ws.ptr(), _stream_ptr(stream)))
 
 
@@ -226,7 +231,7 @@ def quality(x: torch.Tensor, y: torch.Tensor, bound: float = -1.0, out: torch.Te
     _require_cuda(y, "y", torch.float32)
     if x.numel() != y.numel():
         raise ValueError("x and y must have the same number of elements")
-    key = (x.device.index, torch.cuda.current_stream(x.device).cuda_stream)
+    key = (x.device.index, _stream_ptr(stream))            # one quality workspace per stream
     qws = _qws_cache.get(key)
     if qws is None:
         qws = torch.zeros(int(lib().cuszp_quality_workspace_bytes()), dtype=torch.uint8, device=x.device)
