@@ -74,3 +74,22 @@ def test_minmax_and_wrong_L(Lb):
     assert cz.last_status() == cz.ECORRUPT
     with pytest.raises(cz.CuszpError):
         cz.compress(x, 1e-3, "rel", block_len=48)
+
+
+@pytest.mark.parametrize("Lb,order", [(64, 1), (128, 1), (32, 2)])
+def test_empty_tiny_and_nonfinite(Lb, order):
+    for x_np in (np.zeros(0, np.float32), np.array([1.5], np.float32), np.array([1.0, -2.0], np.float32),
+                 np.array([1.0, np.nan, 2.0], np.float32), np.array([np.inf, 0.0], np.float32)):
+        for mode, eb in ((oracle.REL, 1e-3), (oracle.ABS, 1e-2)):
+            st_o, s_o = oracle.compress_ex(x_np, eb, mode, Lb, order)
+            x = torch.from_numpy(x_np).to(DEV)
+            out, nb = cz.compress(x, eb, mode, block_len=Lb, order=order)
+            torch.cuda.synchronize()
+            s_g = out[: int(nb.item())].cpu().numpy()
+            assert s_g[6] == st_o, (Lb, order, x_np, mode, s_g[6], st_o)
+            if st_o == oracle.OK:
+                assert np.array_equal(s_g, s_o), (Lb, order, x_np, mode)
+                y = cz.decompress(out, x_np.size, in_bytes=s_o.size, block_len=Lb, order=order)
+                st, y_o = oracle.decompress(s_o, x_np.size)
+                torch.cuda.synchronize()
+                assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32))
