@@ -93,3 +93,20 @@ def test_empty_tiny_and_nonfinite(Lb, order):
                 st, y_o = oracle.decompress(s_o, x_np.size)
                 torch.cuda.synchronize()
                 assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32))
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("Lb,order", [(64, 1), (128, 1), (32, 2)])
+def test_full_size_nyx(Lb, order):
+    """BASELINE's NYX-shaped 512^3 field (537 MB) at REL 1e-4: whole stream and
+    reconstruction against the oracle for every variant."""
+    x = synth.field_for_config("c4_nyx", device=DEV)
+    x_np = x.cpu().numpy()
+    st, s_o = oracle.compress_ex(x_np, 1e-4, oracle.REL, Lb, order)
+    assert st == oracle.OK
+    out, nb = cz.compress(x, 1e-4, "rel", block_len=Lb, order=order)
+    torch.cuda.synchronize()
+    assert np.array_equal(out[: int(nb.item())].cpu().numpy(), s_o)
+    y = cz.decompress(out, x.numel(), in_bytes=int(nb.item()), block_len=Lb, order=order)
+    st, y_o = oracle.decompress(s_o, x_np.size)
+    assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32))
