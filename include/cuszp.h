@@ -119,14 +119,15 @@ int cuszp_compress_minmax(const float* d_in, size_t n, float lambda,
 int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n,
                      void* d_ws, size_t ws_bytes, void* stream);
 
-/* ---- block-length variants L in {32, 64, 128}
+/* ---- block-length variants L in {8, 16, 32, 64, 128}
  * (the lengths of the paper's smoothness analysis).  Eq 2 is
  * CmpL = (F+1) L/8 bytes; a plane is L/8 bytes with element j at byte j/8,
  * bit j%8 (R9 generalised); header byte 7 = log2(L); one F byte
  * per L-block.  The calls without _L are the L = 32 ones.  Output buffers
  * need cuszp_max_compressed_bytes_L(n, L) bytes (32 + align16(nb) +
  * 32 L/8 nb, nb = ceil(n/L)); workspaces are sized as for L = 32.
- * block_len outside {32, 64, 128}: EINVAL (the size helper returns 0).
+ * block_len outside {8, 16, 32, 64, 128}: EINVAL (the size helper returns 0).
+ * L = 8 / 16 run three launches per call (csrc/small_l.cu); same statuses.
  * Decompression must be given the stream's L (a header with another L:
  * async ECORRUPT). */
 size_t cuszp_max_compressed_bytes_L(size_t n, int block_len);

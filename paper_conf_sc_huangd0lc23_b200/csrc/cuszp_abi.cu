@@ -15,6 +15,9 @@ uint64_t num_blocks(uint64_t n, int L = kL) { return (n + L - 1) / L; }
 // M = L / 32 for the block lengths of SURVEY 8(f) rank 3 (0: unsupported)
 int sub_blocks(int L) { return L == 32 ? 1 : L == 64 ? 2 : L == 128 ? 4 : 0; }
 int mi(int M) { return M == 1 ? 0 : M == 2 ? 1 : 2; }
+// L = 8 / 16: byte-granular planes, the one-thread-per-block path (small_l.cu)
+bool small_L(int L) { return L == 8 || L == 16; }
+bool valid_L(int L) { return sub_blocks(L) != 0 || small_L(L); }
 uint64_t num_tiles(uint64_t n) { return (num_blocks(n) + kTileBlocks - 1) / kTileBlocks; }
 
 struct DeviceInfo {
@@ -71,7 +74,7 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
                     int n_pairs, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
                     void* d_ws, size_t ws_bytes, cudaStream_t stream, int L = kL, int order = 1) {
   const int M = sub_blocks(L);
-  if (M == 0 || (order != 1 && order != 2) || (order == 2 && M != 1)) return CUSZP_EINVAL;
+  if (!valid_L(L) || (order != 1 && order != 2) || (order == 2 && M != 1)) return CUSZP_EINVAL;
   if (out_capacity < cuszp_max_compressed_bytes_L(n, L) || ws_bytes < cuszp_workspace_bytes(n))
     return CUSZP_ENOSPACE;
   DeviceInfo di;
@@ -91,6 +94,7 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
   a.trace = g_trace;
+  if (small_L(L)) return compress_small_launch(L, a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
   const int occ = di.occ_c[mi(M)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;
@@ -105,7 +109,7 @@ extern "C" {
 size_t cuszp_max_compressed_bytes(size_t n) { return cuszp_max_compressed_bytes_L(n, kL); }
 
 size_t cuszp_max_compressed_bytes_L(size_t n, int block_len) {
-  if (sub_blocks(block_len) == 0) return 0;
+  if (!valid_L(block_len)) return 0;
   // a valid block takes at most 25 words (F <= 24, R5); a block of data that
   // fails the guard is only known to be ERANGE at the end of the kernel and
   // may take 32 (v is 32-bit): the bound covers that too (DESIGN 9.5)
@@ -177,7 +181,7 @@ int cuszp_compress_L(const float* d_in, size_t n, float eb, int mode, int block_
 int cuszp_compress_ex(const float* d_in, size_t n, float eb, int mode, int block_len, int order, void* d_out,
                       size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes,
                       void* stream) {
-  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || sub_blocks(block_len) == 0 ||
+  if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || !valid_L(block_len) ||
       (order != 1 && order != 2) || (order == 2 && block_len != kL))
     return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
@@ -215,7 +219,7 @@ int cuszp_compress_minmax_L(const float* d_in, size_t n, float lambda, const flo
                             int block_len, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
                             void* d_ws, size_t ws_bytes, void* stream) {
   if ((n > 0 && d_in == nullptr) || d_out == nullptr || d_ws == nullptr || d_minmax == nullptr ||
-      n_pairs <= 0 || sub_blocks(block_len) == 0)
+      n_pairs <= 0 || !valid_L(block_len))
     return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
       (reinterpret_cast<uintptr_t>(d_ws) & 15u))
@@ -238,7 +242,7 @@ int cuszp_decompress_L(const void* d_in, size_t in_bytes, float* d_out, size_t n
 int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t n, int block_len, int order,
                         void* d_ws, size_t ws_bytes, void* stream) {
   const int M = sub_blocks(block_len);
-  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr || M == 0 ||
+  if (d_in == nullptr || (n > 0 && d_out == nullptr) || d_ws == nullptr || !valid_L(block_len) ||
       (order != 1 && order != 2) || (order == 2 && M != 1))
     return CUSZP_EINVAL;
   if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
@@ -258,6 +262,9 @@ int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t 
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
   a.trace = g_trace;
+  if (small_L(block_len))
+    return decompress_small_launch(block_len, a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK
+                                                                                                : CUSZP_ECUDA;
   const int occ = di.occ_d[mi(M)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (grid > a.num_tiles) grid = a.num_tiles;

@@ -434,6 +434,9 @@ cudaError_t compress_configure(int M, int* occupancy);        // smem attribute 
 cudaError_t compress_launch(int M, int order, unsigned grid, const CompressArgs& a, cudaStream_t s);
 cudaError_t decompress_configure(int M, int* occupancy);
 cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s);
+// L in {8, 16} (small_l.cu): three launches each, one thread per L-block.
+cudaError_t compress_small_launch(int L, const CompressArgs& a, cudaStream_t s);
+cudaError_t decompress_small_launch(int L, const DecompressArgs& a, cudaStream_t s);
 __global__ void quality_kernel(QualityArgs a);
 __global__ void range_kernel(RangeArgs a);
 int launch_copy_len(void* dst, const void* src, const unsigned long long* d_len, uint64_t cap,

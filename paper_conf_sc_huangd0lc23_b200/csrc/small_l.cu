@@ -1,0 +1,395 @@
+// small_l.cu -- block lengths L in {8, 16} (the
+// paper's smoothness analysis spans L = 8..128, Fig 6).
+//
+// At L <= 16 a bit plane is one or two BYTES (R9 generalised),
+// so the word-granular warp transpose of the L >= 32 kernels does not
+// apply.  This path is one thread per L-block, tiles of 4096 elements
+// (the L = 32 tile, so the caller's workspace holds one u64 per tile):
+//   compress:   sizes (quantise, Lorenzo, F, tile byte sums)  ->
+//               tile scan + header (one CTA)                   ->
+//               write (re-quantise, CTA scan of block bytes, sign map + planes)
+//   decompress: sizes (F -> tile byte sums) -> tile scan + header check ->
+//               decode (CTA scan, planes -> |l|, signs, prefix sum, r * 2eb)
+// Three launches each and the input is read twice on compress: a correct
+// first path for the variant, not a tuned one (DESIGN 9.4).
+//
+// Status words: each tile's byte sum / exclusive prefix is stored < 2^40,
+// so its epoch field is 0 and the look-back of the L >= 32 kernels (epochs
+// >= 1) never takes it for a published word.
+#include "internal.cuh"
+
+namespace cuszp {
+namespace {
+
+constexpr int kSThreads = 256;
+constexpr int kSTileElems = 4096;
+constexpr int kScanThreads = 1024;
+
+// eb_abs (Eq 1): ABS -> delta; REL -> lambda * (max - min) over the pairs (R3)
+__device__ __forceinline__ float resolve_eb(const CompressArgs& a) {
+  float eb = a.eb_in;
+  if (a.mode == CUSZP_REL && a.n_pairs == 0) return 0.0f;   // R11
+  if (a.mode == CUSZP_REL) {
+    float mn = a.minmax[0], mx = a.minmax[1];
+    bool nan = isnan(mn) || isnan(mx);
+    for (int p = 1; p < a.n_pairs; ++p) {
+      const float lo = a.minmax[2 * p], hi = a.minmax[2 * p + 1];
+      nan |= isnan(lo) || isnan(hi);
+      if (lo < mn) mn = lo;
+      if (hi > mx) mx = hi;
+    }
+    eb = __fmul_rn(a.eb_in, __fsub_rn(mx, mn));
+    if (nan) eb = __int_as_float(0x7fc00000);
+  }
+  return eb;
+}
+
+__device__ __forceinline__ bool eb_usable(float eb) {
+  return (eb >= kFltMin) && isfinite(__fadd_rn(eb, eb));
+}
+
+// R2: r0 = nearest integer (ties to even) to the exact product d * recip
+// (exact in double), guard |r0| < 2^22 (R5), then the one-step correction
+// that makes |d - r * 2eb| <= eb.  Returns false when the guard fails.
+__device__ __forceinline__ bool quantize(float d, float eb, float two_eb, float recip, int32_t& r) {
+  const double r0d = rint(__dmul_rn(double(d), double(recip)));
+  if (!(fabs(r0d) < double(kGuard))) { r = 0; return false; }
+  const float r0 = float(r0d);
+  const float res = __fmaf_rn(-r0, two_eb, d);
+  r = int32_t(r0) + (res > eb ? 1 : 0) - (res < -eb ? 1 : 0);
+  return true;
+}
+
+// One L-block: Lorenzo residuals l_i = r_i - r_{i-1} (r_{-1} = 0),
+// returns F = bit length of max |l|; *bad on a guard failure.
+template <int L>
+__device__ __forceinline__ int block_encode(const float* in, uint64_t n, uint64_t k, float eb, float two_eb,
+                                            float recip, uint32_t* mag, uint32_t& sign, bool& bad) {
+  int32_t prev = 0;
+  uint32_t mx = 0;
+  sign = 0;
+#pragma unroll
+  for (int i = 0; i < L; ++i) {
+    const uint64_t idx = k * L + uint64_t(i);
+    int32_t r = 0;
+    if (idx < n && !quantize(in[idx], eb, two_eb, recip, r)) bad = true;   // zero pad beyond n (R8)
+    const int32_t l = r - prev;
+    prev = r;
+    if (l < 0) sign |= 1u << i;
+    mag[i] = l < 0 ? uint32_t(-int64_t(l)) : uint32_t(l);
+    mx = max(mx, mag[i]);
+  }
+  return mx == 0 ? 0 : 32 - __clz(int(mx));
+}
+
+// Exclusive CTA scan of one u32 per thread; *total = the CTA sum.
+__device__ __forceinline__ uint32_t cta_excl_scan(uint32_t v, uint32_t* total) {
+  __shared__ uint32_t s_warp[kSThreads / 32];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_warp[warp] = x;
+  __syncthreads();
+  uint32_t base = 0, sum = 0;
+#pragma unroll
+  for (int w = 0; w < kSThreads / 32; ++w) {
+    const uint32_t s = s_warp[w];
+    if (w < warp) base += s;
+    sum += s;
+  }
+  __syncthreads();
+  *total = sum;
+  return base + x - v;
+}
+
+__device__ __forceinline__ uint32_t block_bytes(uint32_t F, int L) { return F == 0 ? 0u : (F + 1u) * uint32_t(L / 8); }
+
+// ---------------------------------------------------------------- compress
+template <int L>
+__global__ void __launch_bounds__(kSThreads) small_sizes_kernel(CompressArgs a) {
+  constexpr int kBlocks = kSTileElems / L;                 // L-blocks per tile
+  static_assert(kBlocks % kSThreads == 0, "tile geometry");
+  const float eb = resolve_eb(a);
+  const bool eb_ok = eb_usable(eb);
+  const float two_eb = __fadd_rn(eb, eb);
+  const float recip = __fdiv_rn(1.0f, two_eb);
+  const uint64_t t = blockIdx.x;
+  uint32_t bytes = 0;
+  bool bad = !eb_ok;
+  if (eb_ok) {
+    for (int j = threadIdx.x; j < kBlocks; j += kSThreads) {
+      const uint64_t k = t * kBlocks + uint64_t(j);
+      if (k >= a.nb) break;
+      uint32_t mag[L], sign;
+      const int F = block_encode<L>(a.in, a.n, k, eb, two_eb, recip, mag, sign, bad);
+      a.out[kHdr + k] = uint8_t(F > kMaxF ? 0 : F);
+      bytes += block_bytes(uint32_t(F), L);
+    }
+  }
+  uint32_t total;
+  cta_excl_scan(bytes, &total);
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(&a.ws->status_accum, kBadRange);
+  if (threadIdx.x == 0) a.status[t] = total;
+}
+
+// One CTA: exclusive scan of the tile byte sums in place, then the header.
+template <int L>
+__global__ void __launch_bounds__(kScanThreads) small_scan_kernel(CompressArgs a) {
+  __shared__ uint64_t s_warp[kScanThreads / 32];
+  __shared__ uint64_t s_carry;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t acc = *reinterpret_cast<volatile uint32_t*>(&a.ws->status_accum);
+  const uint32_t status = (a.n > 0 && (acc & kBadRange)) ? CUSZP_ERANGE : CUSZP_OK;
+  if (threadIdx.x == 0) s_carry = 0;
+  __syncthreads();
+  if (status == CUSZP_OK) {
+    for (uint64_t base = 0; base < a.num_tiles; base += kScanThreads) {
+      const uint64_t i = base + threadIdx.x;
+      const uint64_t v = i < a.num_tiles ? a.status[i] : 0;
+      uint64_t x = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+      }
+      if (lane == 31) s_warp[warp] = x;
+      __syncthreads();
+      uint64_t wb = 0, sum = 0;
+      for (int w = 0; w < kScanThreads / 32; ++w) {
+        if (w < warp) wb += s_warp[w];
+        sum += s_warp[w];
+      }
+      const uint64_t carry = s_carry;
+      if (i < a.num_tiles) a.status[i] = carry + wb + x - v;
+      __syncthreads();
+      if (threadIdx.x == 0) s_carry = carry + sum;
+      __syncthreads();
+    }
+  }
+  if (threadIdx.x < 16 && a.nb + threadIdx.x < align16(a.nb))
+    a.out[kHdr + a.nb + threadIdx.x] = 0;                  // F-area padding (R10)
+  if (threadIdx.x == 0) {
+    const float eb = resolve_eb(a);
+    const uint64_t payload = status == CUSZP_OK ? s_carry : 0;
+    const uint64_t p0 = kHdr + align16(a.nb);
+    uint8_t* h = a.out;                                      // header (R10)
+    *reinterpret_cast<uint32_t*>(h) = 0x505A5343u;           // "CSZP"
+    h[4] = CUSZP_VERSION;
+    h[5] = uint8_t(a.mode);
+    h[6] = uint8_t(status);
+    h[7] = uint8_t(L == 8 ? 3 : 4);                          // log2(L)
+    *reinterpret_cast<uint64_t*>(h + 8) = a.n;
+    *reinterpret_cast<float*>(h + 16) = a.mode == CUSZP_REL ? eb : a.eb_in;
+    *reinterpret_cast<float*>(h + 20) = a.eb_in;
+    *reinterpret_cast<uint64_t*>(h + 24) = payload;
+    if (a.out_bytes) *a.out_bytes = (a.n == 0) ? uint64_t(kHdr) : p0 + payload;
+    a.ws->last_status = status;
+    a.ws->status_accum = 0;
+    __threadfence();
+  }
+}
+
+template <int L>
+__global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) {
+  constexpr int kBlocks = kSTileElems / L;
+  constexpr int kPer = kBlocks / kSThreads;                 // blocks per thread (contiguous)
+  constexpr int kPB = L / 8;                                // bytes per plane
+  if (a.out[6] != CUSZP_OK) return;
+  const float eb = resolve_eb(a);
+  const float two_eb = __fadd_rn(eb, eb);
+  const float recip = __fdiv_rn(1.0f, two_eb);
+  const uint64_t t = blockIdx.x;
+  const uint64_t k0 = t * kBlocks + uint64_t(threadIdx.x) * kPer;
+  uint32_t bytes = 0;
+#pragma unroll
+  for (int j = 0; j < kPer; ++j)
+    if (k0 + j < a.nb) bytes += block_bytes(a.out[kHdr + k0 + j], L);
+  uint32_t total;
+  uint64_t off = kHdr + align16(a.nb) + a.status[t] + cta_excl_scan(bytes, &total);
+  bool bad = false;
+  for (int j = 0; j < kPer; ++j) {
+    const uint64_t k = k0 + j;
+    if (k >= a.nb) break;
+    uint32_t mag[L], sign;
+    const int F = block_encode<L>(a.in, a.n, k, eb, two_eb, recip, mag, sign, bad);
+    if (F == 0) continue;                                   // zero block: F byte only (R6)
+    uint8_t* o = a.out + off;
+#pragma unroll
+    for (int b = 0; b < kPB; ++b) o[b] = uint8_t(sign >> (8 * b));   // sign map (R7, R9)
+    for (int p = 0; p < F; ++p) {                           // block bit-shuffle
+      uint32_t plane = 0;
+#pragma unroll
+      for (int i = 0; i < L; ++i) plane |= ((mag[i] >> p) & 1u) << i;
+#pragma unroll
+      for (int b = 0; b < kPB; ++b) o[kPB * (1 + p) + b] = uint8_t(plane >> (8 * b));
+    }
+    off += block_bytes(uint32_t(F), L);
+  }
+}
+
+// -------------------------------------------------------------- decompress
+template <int L>
+__device__ __forceinline__ uint32_t header_status(const DecompressArgs& a, float* eb_out, uint64_t* pbytes) {
+  const uint64_t p0 = kHdr + align16(a.nb);
+  if (a.in_bytes < uint64_t(kHdr)) return CUSZP_ECORRUPT;
+  const uint8_t* h = a.in;
+  const uint32_t magic = *reinterpret_cast<const uint32_t*>(h);
+  const uint64_t hn = *reinterpret_cast<const uint64_t*>(h + 8);
+  const float eb = *reinterpret_cast<const float*>(h + 16);
+  *pbytes = *reinterpret_cast<const uint64_t*>(h + 24);
+  *eb_out = eb;
+  if (magic != 0x505A5343u || h[4] != CUSZP_VERSION || h[7] != uint8_t(L == 8 ? 3 : 4) || (h[5] & 0x10) != 0)
+    return CUSZP_ECORRUPT;
+  if (h[6] != CUSZP_OK) return h[6] == CUSZP_ERANGE ? CUSZP_ERANGE : CUSZP_ECORRUPT;
+  if (hn != a.n) return CUSZP_EINVAL;
+  if (a.n > 0) {
+    if (!eb_usable(eb)) return CUSZP_ECORRUPT;
+    if (a.in_bytes < p0 || a.in_bytes - p0 < *pbytes) return CUSZP_ECORRUPT;
+  }
+  return CUSZP_OK;
+}
+
+template <int L>
+__global__ void __launch_bounds__(kSThreads) small_dsizes_kernel(DecompressArgs a) {
+  constexpr int kBlocks = kSTileElems / L;
+  float eb;
+  uint64_t pbytes;
+  if (header_status<L>(a, &eb, &pbytes) != CUSZP_OK) return;
+  const uint64_t t = blockIdx.x;
+  uint32_t bytes = 0;
+  bool bad = false;
+  for (int j = threadIdx.x; j < kBlocks; j += kSThreads) {
+    const uint64_t k = t * kBlocks + uint64_t(j);
+    if (k >= a.nb) break;
+    const uint32_t F = a.in[kHdr + k];
+    if (F > uint32_t(kMaxF)) bad = true;
+    else bytes += block_bytes(F, L);
+  }
+  uint32_t total;
+  cta_excl_scan(bytes, &total);
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(&a.ws->status_accum, kBadCorrupt);
+  if (threadIdx.x == 0) a.status[t] = total;
+}
+
+template <int L>
+__global__ void __launch_bounds__(kScanThreads) small_dscan_kernel(DecompressArgs a) {
+  __shared__ uint64_t s_warp[kScanThreads / 32];
+  __shared__ uint64_t s_carry;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  float eb;
+  uint64_t pbytes = 0;
+  uint32_t status = header_status<L>(a, &eb, &pbytes);
+  const uint32_t acc = *reinterpret_cast<volatile uint32_t*>(&a.ws->status_accum);
+  if (status == CUSZP_OK && (acc & kBadCorrupt)) status = CUSZP_ECORRUPT;
+  if (threadIdx.x == 0) s_carry = 0;
+  __syncthreads();
+  if (status == CUSZP_OK && a.n > 0) {
+    for (uint64_t base = 0; base < a.num_tiles; base += kScanThreads) {
+      const uint64_t i = base + threadIdx.x;
+      const uint64_t v = i < a.num_tiles ? a.status[i] : 0;
+      uint64_t x = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+      }
+      if (lane == 31) s_warp[warp] = x;
+      __syncthreads();
+      uint64_t wb = 0, sum = 0;
+      for (int w = 0; w < kScanThreads / 32; ++w) {
+        if (w < warp) wb += s_warp[w];
+        sum += s_warp[w];
+      }
+      const uint64_t carry = s_carry;
+      if (i < a.num_tiles) a.status[i] = carry + wb + x - v;
+      __syncthreads();
+      if (threadIdx.x == 0) s_carry = carry + sum;
+      __syncthreads();
+    }
+    if (s_carry != pbytes) status = CUSZP_ECORRUPT;       // Eq 3 total vs the header
+  }
+  if (threadIdx.x == 0) {
+    a.ws->last_status = status;
+    a.ws->status_accum = 0;
+    __threadfence();
+  }
+}
+
+template <int L>
+__global__ void __launch_bounds__(kSThreads) small_decode_kernel(DecompressArgs a) {
+  constexpr int kBlocks = kSTileElems / L;
+  constexpr int kPer = kBlocks / kSThreads;
+  constexpr int kPB = L / 8;
+  if (*reinterpret_cast<volatile uint32_t*>(&a.ws->last_status) != CUSZP_OK) return;
+  const float eb = *reinterpret_cast<const float*>(a.in + 16);
+  const float two_eb = __fadd_rn(eb, eb);
+  const uint64_t t = blockIdx.x;
+  const uint64_t k0 = t * kBlocks + uint64_t(threadIdx.x) * kPer;
+  uint32_t bytes = 0;
+#pragma unroll
+  for (int j = 0; j < kPer; ++j)
+    if (k0 + j < a.nb) bytes += block_bytes(a.in[kHdr + k0 + j], L);
+  uint32_t total;
+  uint64_t off = kHdr + align16(a.nb) + a.status[t] + cta_excl_scan(bytes, &total);
+  for (int j = 0; j < kPer; ++j) {
+    const uint64_t k = k0 + j;
+    if (k >= a.nb) break;
+    const uint32_t F = a.in[kHdr + k];
+    const uint8_t* p = a.in + off;
+    uint32_t sign = 0;
+    uint32_t mag[L];
+#pragma unroll
+    for (int i = 0; i < L; ++i) mag[i] = 0;
+    if (F > 0) {
+#pragma unroll
+      for (int b = 0; b < kPB; ++b) sign |= uint32_t(p[b]) << (8 * b);
+      for (uint32_t q = 0; q < F; ++q) {
+        uint32_t plane = 0;
+#pragma unroll
+        for (int b = 0; b < kPB; ++b) plane |= uint32_t(p[kPB * (1 + q) + b]) << (8 * b);
+#pragma unroll
+        for (int i = 0; i < L; ++i) mag[i] |= ((plane >> i) & 1u) << q;
+      }
+    }
+    int32_t r = 0;                                         // reverse Lorenzo
+#pragma unroll
+    for (int i = 0; i < L; ++i) {
+      r += ((sign >> i) & 1u) ? -int32_t(mag[i]) : int32_t(mag[i]);
+      const uint64_t idx = k * L + uint64_t(i);
+      if (idx < a.n) a.out[idx] = __fmul_rn(float(r), two_eb);   // d' = r * 2eb
+    }
+    off += block_bytes(F, L);
+  }
+}
+
+template <int L>
+cudaError_t compress_small(const CompressArgs& a, cudaStream_t s) {
+  if (a.num_tiles > 0) small_sizes_kernel<L><<<a.num_tiles, kSThreads, 0, s>>>(a);
+  small_scan_kernel<L><<<1, kScanThreads, 0, s>>>(a);
+  if (a.num_tiles > 0) small_write_kernel<L><<<a.num_tiles, kSThreads, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+template <int L>
+cudaError_t decompress_small(const DecompressArgs& a, cudaStream_t s) {
+  if (a.num_tiles > 0) small_dsizes_kernel<L><<<a.num_tiles, kSThreads, 0, s>>>(a);
+  small_dscan_kernel<L><<<1, kScanThreads, 0, s>>>(a);
+  if (a.num_tiles > 0) small_decode_kernel<L><<<a.num_tiles, kSThreads, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t compress_small_launch(int L, const CompressArgs& a, cudaStream_t s) {
+  return L == 8 ? compress_small<8>(a, s) : compress_small<16>(a, s);
+}
+
+cudaError_t decompress_small_launch(int L, const DecompressArgs& a, cudaStream_t s) {
+  return L == 8 ? decompress_small<8>(a, s) : decompress_small<16>(a, s);
+}
+
+}  // namespace cuszp

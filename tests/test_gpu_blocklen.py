@@ -1,4 +1,4 @@
-"""GPU parity of the block-length variants L in {64, 128} (SURVEY 8(f) NEXT
+"""GPU parity of the block-length variants L in {8, 16, 64, 128} (SURVEY 8(f) NEXT
 rank 3) against oracle.compress_L / oracle.decompress: compressed bytes
 identical, decompressed floats bit-identical, on sizes spanning many tiles
 with ragged tails and on fields that exercise all three packing modes of
@@ -36,7 +36,7 @@ def parity(x_np: np.ndarray, eb: float, mode: int, Lb: int, label=""):
     assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32)), label
 
 
-@pytest.mark.parametrize("Lb", [64, 128])
+@pytest.mark.parametrize("Lb", [8, 16, 64, 128])
 @pytest.mark.parametrize("n", [2, 31, 64, 65, 129, 4096, 4097, 100_003, 1 << 20])
 def test_sizes(Lb, n):
     rng = np.random.default_rng(n)
@@ -45,14 +45,14 @@ def test_sizes(Lb, n):
     parity(x, 1e-3, oracle.REL, Lb, f"L={Lb} n={n}")
 
 
-@pytest.mark.parametrize("Lb", [64, 128])
+@pytest.mark.parametrize("Lb", [8, 16, 64, 128])
 @pytest.mark.parametrize("field,rel", [("U", 1e-2), ("QCLOUD", 1e-3), ("TC", 1e-4)])
 def test_hurricane_fields(Lb, field, rel):
     x = synth.hurricane_like(field, shape=(20, 100, 100), device="cpu").numpy()
     parity(x, rel, oracle.REL, Lb, f"L={Lb} {field}@{rel}")
 
 
-@pytest.mark.parametrize("Lb", [64, 128])
+@pytest.mark.parametrize("Lb", [8, 16, 64, 128])
 def test_wide_fixed_lengths(Lb):
     # ABS with a tiny bound: F up to the guard's 24 bits (one block per transpose)
     rng = np.random.default_rng(Lb)
@@ -61,7 +61,7 @@ def test_wide_fixed_lengths(Lb):
         parity(x, eb, oracle.ABS, Lb, f"L={Lb} abs eb={eb}")
 
 
-@pytest.mark.parametrize("Lb", [64, 128])
+@pytest.mark.parametrize("Lb", [8, 16, 64, 128])
 def test_minmax_and_wrong_L(Lb):
     x_np = synth.smooth1d(200_000, seed=3, device="cpu").numpy()
     x = torch.from_numpy(x_np).to(DEV)
@@ -76,7 +76,7 @@ def test_minmax_and_wrong_L(Lb):
         cz.compress(x, 1e-3, "rel", block_len=48)
 
 
-@pytest.mark.parametrize("Lb,order", [(64, 1), (128, 1), (32, 2)])
+@pytest.mark.parametrize("Lb,order", [(8, 1), (16, 1), (64, 1), (128, 1), (32, 2)])
 def test_empty_tiny_and_nonfinite(Lb, order):
     for x_np in (np.zeros(0, np.float32), np.array([1.5], np.float32), np.array([1.0, -2.0], np.float32),
                  np.array([1.0, np.nan, 2.0], np.float32), np.array([np.inf, 0.0], np.float32)):
@@ -96,7 +96,7 @@ def test_empty_tiny_and_nonfinite(Lb, order):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("Lb,order", [(64, 1), (128, 1), (32, 2)])
+@pytest.mark.parametrize("Lb,order", [(8, 1), (16, 1), (64, 1), (128, 1), (32, 2)])
 def test_full_size_nyx(Lb, order):
     """BASELINE's NYX-shaped 512^3 field (537 MB) at REL 1e-4: whole stream and
     reconstruction against the oracle for every variant."""
@@ -110,3 +110,25 @@ def test_full_size_nyx(Lb, order):
     y = cz.decompress(out, x.numel(), in_bytes=int(nb.item()), block_len=Lb, order=order)
     st, y_o = oracle.decompress(s_o, x_np.size)
     assert np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32))
+
+
+def test_small_L_interleaved_with_word_kernels_and_corrupt_F():
+    """L = 8 / 16 (byte-plane path, small_l.cu) and L = 32 / 64 (look-back
+    kernels) alternate on one workspace: the small path's tile sums must never
+    be read as published look-back words.  A fixed-length byte above 24 in an
+    L = 8 stream is ECORRUPT (as for the oracle)."""
+    rng = np.random.default_rng(11)
+    x_np = np.cumsum(rng.standard_normal(300_001)).astype(np.float32)
+    for Lb in (8, 32, 16, 64, 8, 32):
+        parity(x_np, 1e-3, oracle.REL, Lb, f"interleaved L={Lb}")
+    x = torch.from_numpy(x_np).to(DEV)
+    out, nb = cz.compress(x, 1e-3, "rel", block_len=8)
+    bad = out.clone()
+    bad[32 + 5] = 25
+    st, _ = oracle.decompress(bad[: int(nb.item())].cpu().numpy(), x_np.size)
+    assert st == oracle.ECORRUPT
+    cz.decompress(bad, x_np.size, in_bytes=int(nb.item()), block_len=8)
+    assert cz.last_status() == cz.ECORRUPT
+    y = cz.decompress(out, x_np.size, in_bytes=int(nb.item()), block_len=8)
+    assert cz.last_status() == cz.OK
+    assert torch.max(torch.abs(y - x)).item() <= float(cz.read_header(out)["eb_abs"]) * 1.001
