@@ -65,14 +65,25 @@ __device__ __forceinline__ bool quantize(float d, float eb, float two_eb, float 
 template <int L>
 __device__ __forceinline__ int block_encode(const float* in, uint64_t n, uint64_t k, float eb, float two_eb,
                                             float recip, uint32_t* mag, uint32_t& sign, bool& bad) {
+  float v[L];
+  if ((k + 1) * L <= n) {                                  // whole block: 16-byte loads (in is 16-byte aligned)
+    const float4* p = reinterpret_cast<const float4*>(in + k * L);
+#pragma unroll
+    for (int q = 0; q < L / 4; ++q) {
+      const float4 f = p[q];
+      v[4 * q] = f.x; v[4 * q + 1] = f.y; v[4 * q + 2] = f.z; v[4 * q + 3] = f.w;
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < L; ++i) v[i] = k * L + uint64_t(i) < n ? in[k * L + i] : 0.0f;   // zero pad (R8)
+  }
   int32_t prev = 0;
   uint32_t mx = 0;
   sign = 0;
 #pragma unroll
   for (int i = 0; i < L; ++i) {
-    const uint64_t idx = k * L + uint64_t(i);
     int32_t r = 0;
-    if (idx < n && !quantize(in[idx], eb, two_eb, recip, r)) bad = true;   // zero pad beyond n (R8)
+    if (!quantize(v[i], eb, two_eb, recip, r)) bad = true;
     const int32_t l = r - prev;
     prev = r;
     if (l < 0) sign |= 1u << i;
@@ -106,6 +117,17 @@ __device__ __forceinline__ uint32_t cta_excl_scan(uint32_t v, uint32_t* total) {
   return base + x - v;
 }
 
+// 8x8 bit-matrix transpose: bit p of byte i -> bit i of byte p.  Moves eight
+// planes of eight elements at once (the block bit-shuffle, and its
+// inverse) instead of one bit per instruction.
+__device__ __forceinline__ uint64_t transpose8(uint64_t x) {
+  uint64_t t;
+  t = (x ^ (x >> 7)) & 0x00AA00AA00AA00AAull;  x = x ^ t ^ (t << 7);
+  t = (x ^ (x >> 14)) & 0x0000CCCC0000CCCCull; x = x ^ t ^ (t << 14);
+  t = (x ^ (x >> 28)) & 0x00000000F0F0F0F0ull; x = x ^ t ^ (t << 28);
+  return x;
+}
+
 __device__ __forceinline__ uint32_t block_bytes(uint32_t F, int L) { return F == 0 ? 0u : (F + 1u) * uint32_t(L / 8); }
 
 // ---------------------------------------------------------------- compress
@@ -136,39 +158,52 @@ __global__ void __launch_bounds__(kSThreads) small_sizes_kernel(CompressArgs a) 
   if (threadIdx.x == 0) a.status[t] = total;
 }
 
+// One CTA, in place: exclusive scan of the T tile sums.  Each thread owns a
+// contiguous chunk (its loads are independent, so the whole array is one
+// round of memory latency), chunk sums are scanned across the CTA, then
+// written back as exclusive prefixes.  Returns the total (every thread).
+__device__ __forceinline__ uint64_t tile_scan(uint64_t* st, uint64_t T, uint64_t* s_warp) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint64_t per = (T + kScanThreads - 1) / kScanThreads;
+  const uint64_t b = min(T, per * threadIdx.x), e = min(T, b + per);
+  uint64_t v = 0;
+  for (uint64_t i = b; i < e; ++i) v += st[i];
+  uint64_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_warp[warp] = x;
+  __syncthreads();
+  uint64_t wb = 0, sum = 0;
+  for (int w = 0; w < kScanThreads / 32; ++w) {
+    if (w < warp) wb += s_warp[w];
+    sum += s_warp[w];
+  }
+  uint64_t run = wb + x - v;
+  for (uint64_t i = b; i < e; ++i) {
+    const uint64_t c = st[i];
+    st[i] = run;
+    run += c;
+  }
+  __syncthreads();
+  return sum;
+}
+
 // One CTA: exclusive scan of the tile byte sums in place, then the header.
 template <int L>
 __global__ void __launch_bounds__(kScanThreads) small_scan_kernel(CompressArgs a) {
   __shared__ uint64_t s_warp[kScanThreads / 32];
   __shared__ uint64_t s_carry;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t acc = *reinterpret_cast<volatile uint32_t*>(&a.ws->status_accum);
   const uint32_t status = (a.n > 0 && (acc & kBadRange)) ? CUSZP_ERANGE : CUSZP_OK;
   if (threadIdx.x == 0) s_carry = 0;
   __syncthreads();
   if (status == CUSZP_OK) {
-    for (uint64_t base = 0; base < a.num_tiles; base += kScanThreads) {
-      const uint64_t i = base + threadIdx.x;
-      const uint64_t v = i < a.num_tiles ? a.status[i] : 0;
-      uint64_t x = v;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint64_t y = __shfl_up_sync(kFull, x, o);
-        if (lane >= o) x += y;
-      }
-      if (lane == 31) s_warp[warp] = x;
-      __syncthreads();
-      uint64_t wb = 0, sum = 0;
-      for (int w = 0; w < kScanThreads / 32; ++w) {
-        if (w < warp) wb += s_warp[w];
-        sum += s_warp[w];
-      }
-      const uint64_t carry = s_carry;
-      if (i < a.num_tiles) a.status[i] = carry + wb + x - v;
-      __syncthreads();
-      if (threadIdx.x == 0) s_carry = carry + sum;
-      __syncthreads();
-    }
+    const uint64_t tot = tile_scan(a.status, a.num_tiles, s_warp);
+    if (threadIdx.x == 0) s_carry = tot;
+    __syncthreads();
   }
   if (threadIdx.x < 16 && a.nb + threadIdx.x < align16(a.nb))
     a.out[kHdr + a.nb + threadIdx.x] = 0;                  // F-area padding (R10)
@@ -208,8 +243,9 @@ __global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) 
 #pragma unroll
   for (int j = 0; j < kPer; ++j)
     if (k0 + j < a.nb) bytes += block_bytes(a.out[kHdr + k0 + j], L);
+  __shared__ __align__(16) uint8_t s_pay[kBlocks * kPB * (kMaxF + 1)];   // the tile's payload
   uint32_t total;
-  uint64_t off = kHdr + align16(a.nb) + a.status[t] + cta_excl_scan(bytes, &total);
+  uint32_t off = cta_excl_scan(bytes, &total);
   bool bad = false;
   for (int j = 0; j < kPer; ++j) {
     const uint64_t k = k0 + j;
@@ -217,18 +253,25 @@ __global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) 
     uint32_t mag[L], sign;
     const int F = block_encode<L>(a.in, a.n, k, eb, two_eb, recip, mag, sign, bad);
     if (F == 0) continue;                                   // zero block: F byte only (R6)
-    uint8_t* o = a.out + off;
+    uint8_t* o = s_pay + off;
 #pragma unroll
     for (int b = 0; b < kPB; ++b) o[b] = uint8_t(sign >> (8 * b));   // sign map (R7, R9)
-    for (int p = 0; p < F; ++p) {                           // block bit-shuffle
-      uint32_t plane = 0;
+    for (int g = 0; 8 * g < F; ++g) {                       // block bit-shuffle, 8 planes at a time
 #pragma unroll
-      for (int i = 0; i < L; ++i) plane |= ((mag[i] >> p) & 1u) << i;
+      for (int b = 0; b < kPB; ++b) {                       // elements 8b .. 8b+7 -> byte b of each plane
+        uint64_t x = 0;
 #pragma unroll
-      for (int b = 0; b < kPB; ++b) o[kPB * (1 + p) + b] = uint8_t(plane >> (8 * b));
+        for (int i = 0; i < 8; ++i) x |= uint64_t((mag[8 * b + i] >> (8 * g)) & 0xffu) << (8 * i);
+        x = transpose8(x);
+        const int np = min(8, F - 8 * g);
+        for (int q = 0; q < np; ++q) o[kPB * (1 + 8 * g + q) + b] = uint8_t(x >> (8 * q));
+      }
     }
     off += block_bytes(uint32_t(F), L);
   }
+  __syncthreads();
+  uint8_t* dst = a.out + kHdr + align16(a.nb) + a.status[t];   // coalesced copy-out
+  for (uint32_t i = threadIdx.x; i < total; i += kSThreads) dst[i] = s_pay[i];
 }
 
 // -------------------------------------------------------------- decompress
@@ -279,7 +322,6 @@ template <int L>
 __global__ void __launch_bounds__(kScanThreads) small_dscan_kernel(DecompressArgs a) {
   __shared__ uint64_t s_warp[kScanThreads / 32];
   __shared__ uint64_t s_carry;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   float eb;
   uint64_t pbytes = 0;
   uint32_t status = header_status<L>(a, &eb, &pbytes);
@@ -288,28 +330,9 @@ __global__ void __launch_bounds__(kScanThreads) small_dscan_kernel(DecompressArg
   if (threadIdx.x == 0) s_carry = 0;
   __syncthreads();
   if (status == CUSZP_OK && a.n > 0) {
-    for (uint64_t base = 0; base < a.num_tiles; base += kScanThreads) {
-      const uint64_t i = base + threadIdx.x;
-      const uint64_t v = i < a.num_tiles ? a.status[i] : 0;
-      uint64_t x = v;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint64_t y = __shfl_up_sync(kFull, x, o);
-        if (lane >= o) x += y;
-      }
-      if (lane == 31) s_warp[warp] = x;
-      __syncthreads();
-      uint64_t wb = 0, sum = 0;
-      for (int w = 0; w < kScanThreads / 32; ++w) {
-        if (w < warp) wb += s_warp[w];
-        sum += s_warp[w];
-      }
-      const uint64_t carry = s_carry;
-      if (i < a.num_tiles) a.status[i] = carry + wb + x - v;
-      __syncthreads();
-      if (threadIdx.x == 0) s_carry = carry + sum;
-      __syncthreads();
-    }
+    const uint64_t tot = tile_scan(a.status, a.num_tiles, s_warp);
+    if (threadIdx.x == 0) s_carry = tot;
+    __syncthreads();
     if (s_carry != pbytes) status = CUSZP_ECORRUPT;       // Eq 3 total vs the header
   }
   if (threadIdx.x == 0) {
@@ -333,13 +356,17 @@ __global__ void __launch_bounds__(kSThreads) small_decode_kernel(DecompressArgs 
 #pragma unroll
   for (int j = 0; j < kPer; ++j)
     if (k0 + j < a.nb) bytes += block_bytes(a.in[kHdr + k0 + j], L);
+  __shared__ __align__(16) uint8_t s_pay[kBlocks * kPB * (kMaxF + 1)];
   uint32_t total;
-  uint64_t off = kHdr + align16(a.nb) + a.status[t] + cta_excl_scan(bytes, &total);
+  uint32_t off = cta_excl_scan(bytes, &total);
+  const uint8_t* src = a.in + kHdr + align16(a.nb) + a.status[t];   // coalesced copy-in
+  for (uint32_t i = threadIdx.x; i < total; i += kSThreads) s_pay[i] = src[i];
+  __syncthreads();
   for (int j = 0; j < kPer; ++j) {
     const uint64_t k = k0 + j;
     if (k >= a.nb) break;
     const uint32_t F = a.in[kHdr + k];
-    const uint8_t* p = a.in + off;
+    const uint8_t* p = s_pay + off;
     uint32_t sign = 0;
     uint32_t mag[L];
 #pragma unroll
@@ -347,20 +374,33 @@ __global__ void __launch_bounds__(kSThreads) small_decode_kernel(DecompressArgs 
     if (F > 0) {
 #pragma unroll
       for (int b = 0; b < kPB; ++b) sign |= uint32_t(p[b]) << (8 * b);
-      for (uint32_t q = 0; q < F; ++q) {
-        uint32_t plane = 0;
+      for (int g = 0; 8 * g < int(F); ++g) {                // inverse bit-shuffle, 8 planes at a time
+        const int np = min(8, int(F) - 8 * g);
 #pragma unroll
-        for (int b = 0; b < kPB; ++b) plane |= uint32_t(p[kPB * (1 + q) + b]) << (8 * b);
+        for (int b = 0; b < kPB; ++b) {
+          uint64_t x = 0;
+          for (int q = 0; q < np; ++q) x |= uint64_t(p[kPB * (1 + 8 * g + q) + b]) << (8 * q);
+          x = transpose8(x);
 #pragma unroll
-        for (int i = 0; i < L; ++i) mag[i] |= ((plane >> i) & 1u) << q;
+          for (int i = 0; i < 8; ++i) mag[8 * b + i] |= uint32_t((x >> (8 * i)) & 0xffu) << (8 * g);
+        }
       }
     }
     int32_t r = 0;                                         // reverse Lorenzo
+    float y[L];
 #pragma unroll
     for (int i = 0; i < L; ++i) {
       r += ((sign >> i) & 1u) ? -int32_t(mag[i]) : int32_t(mag[i]);
-      const uint64_t idx = k * L + uint64_t(i);
-      if (idx < a.n) a.out[idx] = __fmul_rn(float(r), two_eb);   // d' = r * 2eb
+      y[i] = __fmul_rn(float(r), two_eb);                  // d' = r * 2eb
+    }
+    if ((k + 1) * L <= a.n) {                              // whole block: 16-byte stores
+      float4* o = reinterpret_cast<float4*>(a.out + k * L);
+#pragma unroll
+      for (int q = 0; q < L / 4; ++q) o[q] = make_float4(y[4 * q], y[4 * q + 1], y[4 * q + 2], y[4 * q + 3]);
+    } else {
+#pragma unroll
+      for (int i = 0; i < L; ++i)
+        if (k * L + uint64_t(i) < a.n) a.out[k * L + i] = y[i];
     }
     off += block_bytes(F, L);
   }
