@@ -48,13 +48,15 @@ __device__ __forceinline__ bool eb_usable(float eb) {
   return (eb >= kFltMin) && isfinite(__fadd_rn(eb, eb));
 }
 
-// R2: r0 = nearest integer (ties to even) to the exact product d * recip
-// (exact in double), guard |r0| < 2^22 (R5), then the one-step correction
-// that makes |d - r * 2eb| <= eb.  Returns false when the guard fails.
+// R2: r0 = nearest integer (ties to even) to the exact product d * recip,
+// guard |r0| < 2^22 (R5), then the one-step correction that makes
+// |d - r * 2eb| <= eb.  fma(d, recip, 1.5*2^23) rounds the exact product to
+// an integer in ONE rounding while |d * recip| < 2^22, and every product at
+// or beyond that fails the guard either way (DESIGN 8, the fast kernels'
+// sequence).  Returns false when the guard fails (NaN and Inf included).
 __device__ __forceinline__ bool quantize(float d, float eb, float two_eb, float recip, int32_t& r) {
-  const double r0d = rint(__dmul_rn(double(d), double(recip)));
-  if (!(fabs(r0d) < double(kGuard))) { r = 0; return false; }
-  const float r0 = float(r0d);
+  const float r0 = __fsub_rn(__fmaf_rn(d, recip, kRoundMagic), kRoundMagic);
+  if (!(fabsf(r0) < kGuard)) { r = 0; return false; }
   const float res = __fmaf_rn(-r0, two_eb, d);
   r = int32_t(r0) + (res > eb ? 1 : 0) - (res < -eb ? 1 : 0);
   return true;
