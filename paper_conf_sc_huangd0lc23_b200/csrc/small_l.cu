@@ -245,9 +245,11 @@ __global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) 
 #pragma unroll
   for (int j = 0; j < kPer; ++j)
     if (k0 + j < a.nb) bytes += block_bytes(a.out[kHdr + k0 + j], L);
-  __shared__ __align__(16) uint8_t s_pay[kBlocks * kPB * (kMaxF + 1)];   // the tile's payload
+  __shared__ __align__(16) uint8_t s_pay[kBlocks * kPB * (kMaxF + 1) + 16];   // the tile's payload
+  uint8_t* dst = a.out + kHdr + align16(a.nb) + a.status[t];
+  const uint32_t mis = uint32_t(reinterpret_cast<uintptr_t>(dst) & 3u);   // staged at dst's word phase
   uint32_t total;
-  uint32_t off = cta_excl_scan(bytes, &total);
+  uint32_t off = mis + cta_excl_scan(bytes, &total);
   bool bad = false;
   for (int j = 0; j < kPer; ++j) {
     const uint64_t k = k0 + j;
@@ -272,8 +274,18 @@ __global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) 
     off += block_bytes(uint32_t(F), L);
   }
   __syncthreads();
-  uint8_t* dst = a.out + kHdr + align16(a.nb) + a.status[t];   // coalesced copy-out
-  for (uint32_t i = threadIdx.x; i < total; i += kSThreads) dst[i] = s_pay[i];
+  // coalesced copy-out in words; the two edge words are shared with the
+  // neighbouring tiles and go byte by byte
+  uint8_t* dst_al = dst - mis;
+  const uint32_t end = mis + total, nw = (end + 3) / 4;
+  for (uint32_t w = threadIdx.x; w < nw; w += kSThreads) {
+    if (4 * w >= mis && 4 * w + 4 <= end) {
+      reinterpret_cast<uint32_t*>(dst_al)[w] = reinterpret_cast<const uint32_t*>(s_pay)[w];
+    } else {
+      for (uint32_t i = 4 * w; i < 4 * w + 4; ++i)
+        if (i >= mis && i < end) dst_al[i] = s_pay[i];
+    }
+  }
 }
 
 // -------------------------------------------------------------- decompress
@@ -358,11 +370,16 @@ __global__ void __launch_bounds__(kSThreads) small_decode_kernel(DecompressArgs 
 #pragma unroll
   for (int j = 0; j < kPer; ++j)
     if (k0 + j < a.nb) bytes += block_bytes(a.in[kHdr + k0 + j], L);
-  __shared__ __align__(16) uint8_t s_pay[kBlocks * kPB * (kMaxF + 1)];
+  __shared__ __align__(16) uint8_t s_pay[kBlocks * kPB * (kMaxF + 1) + 16];
+  const uint8_t* src = a.in + kHdr + align16(a.nb) + a.status[t];
+  const uint32_t mis = uint32_t(reinterpret_cast<uintptr_t>(src) & 3u);
   uint32_t total;
-  uint32_t off = cta_excl_scan(bytes, &total);
-  const uint8_t* src = a.in + kHdr + align16(a.nb) + a.status[t];   // coalesced copy-in
-  for (uint32_t i = threadIdx.x; i < total; i += kSThreads) s_pay[i] = src[i];
+  uint32_t off = mis + cta_excl_scan(bytes, &total);
+  // coalesced copy-in of whole aligned words (the edge words' extra bytes lie
+  // in the same 4-byte word of the stream, so in the same allocation)
+  const uint32_t nw = (mis + total + 3) / 4;
+  const uint32_t* src_al = reinterpret_cast<const uint32_t*>(src - mis);
+  for (uint32_t w = threadIdx.x; w < nw; w += kSThreads) reinterpret_cast<uint32_t*>(s_pay)[w] = src_al[w];
   __syncthreads();
   for (int j = 0; j < kPer; ++j) {
     const uint64_t k = k0 + j;
