@@ -374,7 +374,7 @@ def run_ours(args, rank, world, dev):
     x0, n0 = xs[f0], n_of[f0]
     cz.check(lib.cuszp_range(x0.data_ptr(), n0, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
     variants = {}
-    for Lb, order in ((32, 1), (64, 1), (128, 1), (32, 2)):
+    for Lb, order in ((8, 1), (16, 1), (32, 1), (64, 1), (128, 1), (32, 2)):
         tc, td = [], []
         capL = cz.max_compressed_bytes(n0, Lb)
         outL = out if capL <= cap else torch.empty(capL, dtype=torch.uint8, device=dev)
