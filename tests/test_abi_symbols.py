@@ -104,8 +104,9 @@ def test_binding_rejects_cpu_tensors():
 
 def test_max_compressed_bytes_L_matches_oracle():
     h = _lib.lib()
-    for Lb in (32, 64, 128):
+    for Lb in (8, 16, 32, 64, 128):
         for n in (0, 1, 2, 31, 64, 129, 10**6 + 3):
             nb = (n + Lb - 1) // Lb
             assert h.cuszp_max_compressed_bytes_L(n, Lb) == oracle.max_compressed_bytes_L(n, Lb) + Lb // 8 * 7 * nb
-    assert h.cuszp_max_compressed_bytes_L(100, 48) == 0
+    for bad in (0, 4, 24, 48, 256):
+        assert h.cuszp_max_compressed_bytes_L(100, bad) == 0
