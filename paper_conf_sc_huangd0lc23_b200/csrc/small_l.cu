@@ -64,11 +64,10 @@ __device__ __forceinline__ bool quantize(float d, float eb, float two_eb, float 
 
 // One L-block: Lorenzo residuals l_i = r_i - r_{i-1} (r_{-1} = 0),
 // returns F = bit length of max |l|; *bad on a guard failure.
+// The L values of block k (zero pad beyond n, R8); whole blocks as float4.
 template <int L>
-__device__ __forceinline__ int block_encode(const float* in, uint64_t n, uint64_t k, float eb, float two_eb,
-                                            float recip, uint32_t* mag, uint32_t& sign, bool& bad) {
-  float v[L];
-  if ((k + 1) * L <= n) {                                  // whole block: 16-byte loads (in is 16-byte aligned)
+__device__ __forceinline__ void block_load(const float* in, uint64_t n, uint64_t k, float* v) {
+  if ((k + 1) * L <= n) {                                  // in is 16-byte aligned (ABI)
     const float4* p = reinterpret_cast<const float4*>(in + k * L);
 #pragma unroll
     for (int q = 0; q < L / 4; ++q) {
@@ -77,8 +76,15 @@ __device__ __forceinline__ int block_encode(const float* in, uint64_t n, uint64_
     }
   } else {
 #pragma unroll
-    for (int i = 0; i < L; ++i) v[i] = k * L + uint64_t(i) < n ? in[k * L + i] : 0.0f;   // zero pad (R8)
+    for (int i = 0; i < L; ++i) v[i] = k * L + uint64_t(i) < n ? in[k * L + i] : 0.0f;
   }
+}
+
+// One L-block: Lorenzo residuals l_i = r_i - r_{i-1} (r_{-1} = 0),
+// returns F = bit length of max |l|; *bad on a guard failure.
+template <int L>
+__device__ __forceinline__ int block_encode(const float* v, float eb, float two_eb, float recip, uint32_t* mag,
+                                            uint32_t& sign, bool& bad) {
   int32_t prev = 0;
   uint32_t mx = 0;
   sign = 0;
@@ -145,11 +151,19 @@ __global__ void __launch_bounds__(kSThreads) small_sizes_kernel(CompressArgs a) 
   uint32_t bytes = 0;
   bool bad = !eb_ok;
   if (eb_ok) {
-    for (int j = threadIdx.x; j < kBlocks; j += kSThreads) {
-      const uint64_t k = t * kBlocks + uint64_t(j);
+    constexpr int kPer = kBlocks / kSThreads;
+    float v[kPer][L];
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {                        // every load in flight before any math
+      const uint64_t k = t * kBlocks + uint64_t(threadIdx.x + j * kSThreads);
+      if (k < a.nb) block_load<L>(a.in, a.n, k, v[j]);
+    }
+#pragma unroll
+    for (int j = 0; j < kPer; ++j) {
+      const uint64_t k = t * kBlocks + uint64_t(threadIdx.x + j * kSThreads);
       if (k >= a.nb) break;
       uint32_t mag[L], sign;
-      const int F = block_encode<L>(a.in, a.n, k, eb, two_eb, recip, mag, sign, bad);
+      const int F = block_encode<L>(v[j], eb, two_eb, recip, mag, sign, bad);
       a.out[kHdr + k] = uint8_t(F > kMaxF ? 0 : F);
       bytes += block_bytes(uint32_t(F), L);
     }
@@ -241,6 +255,10 @@ __global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) 
   const float recip = __fdiv_rn(1.0f, two_eb);
   const uint64_t t = blockIdx.x;
   const uint64_t k0 = t * kBlocks + uint64_t(threadIdx.x) * kPer;
+  float v[kPer][L];                                         // input loads in flight during the scan
+#pragma unroll
+  for (int j = 0; j < kPer; ++j)
+    if (k0 + j < a.nb) block_load<L>(a.in, a.n, k0 + j, v[j]);
   uint32_t bytes = 0;
 #pragma unroll
   for (int j = 0; j < kPer; ++j)
@@ -255,7 +273,7 @@ __global__ void __launch_bounds__(kSThreads) small_write_kernel(CompressArgs a) 
     const uint64_t k = k0 + j;
     if (k >= a.nb) break;
     uint32_t mag[L], sign;
-    const int F = block_encode<L>(a.in, a.n, k, eb, two_eb, recip, mag, sign, bad);
+    const int F = block_encode<L>(v[j], eb, two_eb, recip, mag, sign, bad);
     if (F == 0) continue;                                   // zero block: F byte only (R6)
     uint8_t* o = s_pay + off;
 #pragma unroll
