@@ -186,9 +186,12 @@ int cuszp_decompress_host(const void* h_in, size_t in_bytes, float* h_out, size_
  * ENOSPACE); *h_out_bytes receives the stream length when the stream
  * completes.  decompress: the stream's length is taken from its own header
  * (at most in_capacity bytes are read; d_in_scratch holds in_capacity).
- * Sync errors: EINVAL (NULL or unmapped buffers), ENOSPACE, ECUDA; data
- * errors are asynchronous as for the device calls.  One workspace per
- * stream. */
+ * Alignment: h_out, h_in (mapped sides) and both device scratch buffers
+ * 16-byte aligned, h_out_bytes 8-byte aligned (the copy kernels move 16-
+ * and 8-byte words); checked before anything is launched.
+ * Sync errors: EINVAL (NULL, unmapped or misaligned buffers), ENOSPACE,
+ * ECUDA -- on a sync error nothing has been launched; data errors are
+ * asynchronous as for the device calls.  One workspace per stream. */
 int cuszp_compress_host_async(const float* h_in, size_t n, float eb, int mode,
                               void* h_out, size_t out_capacity, unsigned long long* h_out_bytes,
                               float* d_in_scratch, void* d_out_scratch,

@@ -44,6 +44,12 @@ def _stream_ptr(stream) -> int:
     return int(s.cuda_stream)
 
 
+def _check_out_bytes(t: torch.Tensor):
+    _require_cuda(t, "out_bytes", torch.int64)
+    if t.numel() < 1:
+        raise ValueError("out_bytes must hold one int64")
+
+
 def _require_cuda(t: torch.Tensor, name: str, dtype=None):
     if not isinstance(t, torch.Tensor) or not t.is_cuda:
         raise TypeError(f"{name} must be a CUDA tensor (no CPU path exists)")
@@ -100,9 +106,16 @@ def _workspace(n: int, device, ws: Workspace | None, stream=None) -> Workspace:
     key = (dev_index, int(s.cuda_stream))
     w = _ws_cache.get(key)
     if w is None or not w.fits(n):
+        cur = torch.cuda.current_stream(torch.device("cuda", dev_index))
+        if w is not None:
+            # calls already queued on s may still use the old buffer: the
+            # caching allocator must not hand it out before s reaches this point
+            w.buf.record_stream(s)
         w = Workspace(max(int(n), 1 << 20), device)
         _ws_cache[key] = w
-        s.wait_stream(torch.cuda.current_stream(torch.device("cuda", dev_index)))   # zeroed before first use
+        s.wait_stream(cur)                                   # zeroed (on cur) before first use on s
+        if s != cur:
+            w.buf.record_stream(s)
     return w
 
 
@@ -112,6 +125,9 @@ def value_range(x: torch.Tensor, ws: Workspace | None = None, out: torch.Tensor 
     ws = _workspace(x.numel(), x.device, ws, stream)
     if out is None:
         out = torch.empty(2, dtype=torch.float32, device=x.device)
+    _require_cuda(out, "out", torch.float32)
+    if out.numel() < 2:
+        raise ValueError("out must hold 2 float32 values (min, max)")
     check(lib().cuszp_range(x.data_ptr(), x.numel(), out.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)),
           "cuszp_range")
     return out
@@ -131,6 +147,7 @@ def compress(x: torch.Tensor, eb: float, mode="rel", out: torch.Tensor | None = 
     _require_cuda(out, "out", torch.uint8)
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    _check_out_bytes(out_bytes)
     ws = _workspace(n, x.device, ws, stream)
     check(lib().cuszp_compress_ex(x.data_ptr(), n, float(eb), _mode(mode), int(block_len), int(order),
                                   out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
@@ -147,8 +164,12 @@ def compress_minmax(x: torch.Tensor, lam: float, minmax: torch.Tensor, out: torc
     n = x.numel()
     if out is None:
         out = torch.empty(max_compressed_bytes(n, block_len), dtype=torch.uint8, device=x.device)
+    _require_cuda(out, "out", torch.uint8)
     if out_bytes is None:
         out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    _check_out_bytes(out_bytes)
+    if minmax.numel() < 2:
+        raise ValueError("minmax must hold at least one (min, max) pair")
     ws = _workspace(n, x.device, ws, stream)
     check(lib().cuszp_compress_minmax_L(x.data_ptr(), n, float(lam), minmax.data_ptr(), minmax.numel() // 2,
                                         int(block_len), out.data_ptr(), out.numel(), out_bytes.data_ptr(), ws.ptr(),
@@ -163,8 +184,12 @@ def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None
     if out is None:
         out = torch.empty(int(n), dtype=torch.float32, device=stream_buf.device)
     _require_cuda(out, "out", torch.float32)
+    if out.numel() < int(n):
+        raise ValueError(f"out holds {out.numel()} floats, {int(n)} needed")
     ws = _workspace(n, stream_buf.device, ws, stream)
     nbytes = stream_buf.numel() if in_bytes is None else int(in_bytes)
+    if nbytes > stream_buf.numel() or nbytes < 0:
+        raise ValueError(f"in_bytes={nbytes} exceeds the stream buffer ({stream_buf.numel()} bytes)")
     check(lib().cuszp_decompress_ex(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), int(block_len),
                                     int(order), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_decompress")
     return out
@@ -236,8 +261,16 @@ def quality(x: torch.Tensor, y: torch.Tensor, bound: float = -1.0, out: torch.Te
     if qws is None:
         qws = torch.zeros(int(lib().cuszp_quality_workspace_bytes()), dtype=torch.uint8, device=x.device)
         _qws_cache[key] = qws
+        if stream is not None:
+            cur = torch.cuda.current_stream(x.device)
+            stream.wait_stream(cur)                          # the zeroing (on cur) precedes the first use
+            if stream != cur:
+                qws.record_stream(stream)
     if out is None:
         out = torch.empty(14, dtype=torch.float64, device=x.device)
+    _require_cuda(out, "out", torch.float64)
+    if out.numel() < 14:
+        raise ValueError("out must hold 14 float64 values (cuszp_quality_stats)")
     check(lib().cuszp_quality(x.data_ptr(), y.data_ptr(), x.numel(), float(bound), out.data_ptr(), qws.data_ptr(),
                               qws.numel(), _stream_ptr(stream)), "cuszp_quality")
     if not sync:

@@ -4,8 +4,9 @@
 // Persistent, warp-specialised CTA:
 //   warp 0      producer: takes a tile ticket, streams the tile's 16 KB of
 //               fp32 HBM -> shared memory with one 1D TMA bulk copy
-//               (UBLKCP) into a 3-stage mbarrier ring;
-//   warps 2..9  compute: 16 L-blocks each, one lane per element:
+//               (UBLKCP) into a kStages-deep mbarrier ring;
+//   warps 1..kWriters  writers (below);
+//   warps kWriters+1..  compute (kCW warps): 128/kCW L-blocks each, one lane per element:
 //     a2 pre-quantisation   r = round(d / 2eb)            (R2)
 //     a3 block Lorenzo      l_j = r_j - r_{j-1}, r_{-1}=0
 //     a4 sign map + a8 bit-shuffle: v_j = 2|l_j| + [l_j<0]; a warp bit
@@ -18,7 +19,7 @@
 //     each compute warp appends its words to its own shared-memory ring;
 //     the last compute warp to finish a tile publishes the tile aggregate
 //     (a7, first half of the decoupled look-back) at once;
-//   warps 1..4  writers, tiles round-robin: resolve the tile's prefix by
+//   writers, tiles round-robin: resolve the tile's prefix by
 //               look-back (a7, Eq 3), copy the ring segments to
 //               their global offsets and release ring space in tile order.
 //               Up to kMeta tiles wait for their prefix while the compute

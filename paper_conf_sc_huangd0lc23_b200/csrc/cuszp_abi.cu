@@ -55,6 +55,8 @@ int device_info(DeviceInfo* out) {
   return CUSZP_OK;
 }
 
+bool misaligned(const void* p, uintptr_t a) { return (reinterpret_cast<uintptr_t>(p) & (a - 1)) != 0; }
+
 bool eb_is_normal(float eb) {
   if (!(eb >= kFltMin)) return false;
   const float two = eb + eb;
@@ -353,7 +355,15 @@ int cuszp_compress_host_async(const float* h_in, size_t n, float eb, int mode, v
                               size_t ws_bytes, void* stream) {
   if ((n > 0 && (h_in == nullptr || d_in_scratch == nullptr)) || d_out_scratch == nullptr || d_ws == nullptr)
     return CUSZP_EINVAL;
+  // every check precedes the first launch: the copy kernel moves
+  // 16-byte words into h_out and an 8-byte length into h_out_bytes
+  if (misaligned(h_out, 16) || misaligned(h_out_bytes, 8) || misaligned(d_in_scratch, 16) ||
+      misaligned(d_out_scratch, 16) || misaligned(d_ws, 16))
+    return CUSZP_EINVAL;
   if (out_capacity < cuszp_max_compressed_bytes(n)) return CUSZP_ENOSPACE;
+  if (ws_bytes < cuszp_workspace_bytes(n)) return CUSZP_ENOSPACE;
+  if (mode == CUSZP_ABS ? !eb_is_normal(eb) : (mode != CUSZP_REL || !(eb > 0.0f) || !(eb - eb == 0.0f)))
+    return CUSZP_EINVAL;
   void* out_dev = mapped(h_out);
   unsigned long long* len_dev = static_cast<unsigned long long*>(mapped(h_out_bytes));
   if (out_dev == nullptr || len_dev == nullptr) return CUSZP_EINVAL;
@@ -376,6 +386,11 @@ int cuszp_decompress_host_async(const void* h_in, size_t in_capacity, float* h_o
       (n > 0 && (h_out == nullptr || d_out_scratch == nullptr)))
     return CUSZP_EINVAL;
   if (in_capacity < size_t(kHdr)) return CUSZP_EINVAL;
+  // every check precedes the first launch: the copy kernel reads
+  // 16-byte words of h_in and writes them into d_in_scratch
+  if (misaligned(h_in, 16) || misaligned(d_in_scratch, 16) || misaligned(d_out_scratch, 16) || misaligned(d_ws, 16))
+    return CUSZP_EINVAL;
+  if (ws_bytes < cuszp_workspace_bytes(n)) return CUSZP_ENOSPACE;
   const void* in_dev = mapped(h_in);
   if (in_dev == nullptr) return CUSZP_EINVAL;
   DeviceInfo di;

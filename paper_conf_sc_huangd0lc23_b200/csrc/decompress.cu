@@ -10,7 +10,7 @@
 //               Eq 3) -- one look-back per 4 tiles, overlapped with decoding
 //               through a double-buffered chunk descriptor;
 //   warp 1      loader: streams every tile's payload HBM -> shared memory
-//               with one 1D TMA bulk copy into a 4-stage ring;
+//               with one 1D TMA bulk copy into a kDStages-deep ring;
 //   warps 2..9  compute, 16 blocks each in groups of 4 -- four, two or one
 //               blocks per warp bit transpose (8, 16 or 32 lanes per block):
 //     a10 inverse bit-shuffle: lane k of a block's lane range <- word k

@@ -7,7 +7,7 @@
 // mbarrier ring; compute warps own 16 blocks each with one lane per element
 // (lane j <-> element j), so the paper's per-block steps become warp
 // primitives (Lorenzo = shfl_up, max = redux.max, F = clz, bit-shuffle =
-// a 15-instruction warp bit-transpose that handles two blocks at once); a
+// a 13-instruction warp bit-transpose that handles 1, 2 or 4 blocks at once); a
 // scan warp places each tile with a decoupled look-back (the paper's
 // chained scan) over epoch-tagged status words, so no memset is
 // needed between calls and the look-back latency overlaps the next tile.

@@ -393,11 +393,15 @@ __global__ void __launch_bounds__(kSThreads) small_decode_kernel(DecompressArgs 
   const uint32_t mis = uint32_t(reinterpret_cast<uintptr_t>(src) & 3u);
   uint32_t total;
   uint32_t off = mis + cta_excl_scan(bytes, &total);
-  // coalesced copy-in of whole aligned words (the edge words' extra bytes lie
-  // in the same 4-byte word of the stream, so in the same allocation)
-  const uint32_t nw = (mis + total + 3) / 4;
+  // coalesced copy-in of whole aligned words; the leading edge word's extra
+  // bytes precede this tile's payload inside the stream, the trailing edge
+  // word is copied byte by byte so no read passes the tile's last byte (the
+  // stream may end there: in_bytes bounds every read, cuszp.h)
+  const uint32_t end = mis + total;
+  const uint32_t nfull = end / 4;
   const uint32_t* src_al = reinterpret_cast<const uint32_t*>(src - mis);
-  for (uint32_t w = threadIdx.x; w < nw; w += kSThreads) reinterpret_cast<uint32_t*>(s_pay)[w] = src_al[w];
+  for (uint32_t w = threadIdx.x; w < nfull; w += kSThreads) reinterpret_cast<uint32_t*>(s_pay)[w] = src_al[w];
+  if (threadIdx.x < (end & 3u)) s_pay[4 * nfull + threadIdx.x] = (src - mis)[4 * nfull + threadIdx.x];
   __syncthreads();
   for (int j = 0; j < kPer; ++j) {
     const uint64_t k = k0 + j;
