@@ -123,9 +123,11 @@ int oracle_compress_ex(const float* x, uint64_t n, float eb, int mode, int L, in
  * max_abs_err, max_rel_err, max_pw_rel_err, mse, psnr, nrmse, norm_err,
  * norm_err_norm, pearson; out_counts[0..1] = n, #{|x_i - y_i| > bound}.
  * n must be > 0.  Pinned by the artifact's printed values, closed forms and
- * numpy's corrcoef -- except norm_err_norm (= ||e||/||x||, reading Q2 of
- * "parity unpinned" for that one field, the paper prints it
- * without the data needed to check the normalisation). */
+ * numpy's corrcoef; norm_err_norm (= ||e||_2 / ||x||_2, reading Q2 of
+ * DESIGN.md 9.2) by hand-computed closed forms and by the printed triple
+ * (normErr, normErr_norm, pearson): the printed Pearson coefficient rules out
+ * a centred normalisation, and an input with the printed RMSE and Pearson
+ * coefficient reproduces the printed 0.015479 (tests/test_oracle_quality.py). */
 void oracle_quality(const float* x, const float* y, uint64_t n, double bound,
                     double out[12], uint64_t out_counts[2]);
 

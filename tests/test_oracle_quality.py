@@ -113,3 +113,66 @@ def test_round_trip_bound_count_matches_bruteforce():
     brute = int(np.count_nonzero(np.abs(x.astype(np.float64) - y.astype(np.float64)) > float(eb)))
     assert q["n_over_bound"] == brute
     assert q["max_abs_err"] <= float(eb) + float(np.spacing(np.abs(x)).max())
+
+
+# ---- normErr_norm: the normalisation is fixed by the printed output
+P_NORM_ERR_NORM = 0.015479
+P_PEARSON = 0.999845
+
+
+def test_norm_err_norm_reading_forced_by_printed_pearson():
+    """Which norm divides normErr?  For ANY x, y: var(x - y) >= var(x) (1 - r^2)
+    (minimise sigma_x^2 + sigma_y^2 - 2 r sigma_x sigma_y over sigma_y), so a
+    CENTRED normalisation ||e|| / ||x - mean(x)|| >= sqrt(1 - r^2); with the
+    printed r = 0.999845 that bound is 0.0176 > the printed 0.015479: the
+    centred reading is impossible.  The range-based one is NRMSE (5.77e-5),
+    also not the printed value.  The reading ||e||_2 / ||x||_2 needs
+    RMS(x) = normErr / normErr_norm / sqrt(n) between sigma_x and max|x| --
+    consistent (checked with the construction below)."""
+    lower_centred = math.sqrt(1 - P_PEARSON ** 2)
+    assert lower_centred > P_NORM_ERR_NORM * 1.1
+    assert abs(P_NRMSE - P_NORM_ERR_NORM) > 0.01
+    rms_x = P_NORM_ERR / P_NORM_ERR_NORM / math.sqrt(P_N)
+    assert P_MIN < rms_x < P_MAX
+
+
+def test_oracle_reproduces_printed_norm_err_norm_and_pearson():
+    """An input with the printed RMSE, Pearson coefficient and normErr_norm
+    under the ||x||_2 reading: x = mu + s z, e = d w with z, w = +-1 patterns
+    orthogonal to each other and to 1 (mean error 0, cov(x, e) = 0), so
+    r = s / sqrt(s^2 + d^2) and normErr_norm = d / sqrt(mu^2 + s^2).  The
+    oracle must print both values back to the paper's 6 digits."""
+    n = 1 << 16
+    d = 0.25 * round(P_NRMSE * P_RANGE * 4)                    # 276.0, exact in fp32 arithmetic below
+    s = d * P_PEARSON / math.sqrt(1 - P_PEARSON ** 2)
+    rms = d / P_NORM_ERR_NORM
+    mu = math.sqrt(rms * rms - s * s)
+    s, mu = float(np.float32(s)), float(np.float32(mu))
+    i = np.arange(n)
+    z = np.where((i // 2) % 2 == 0, 1.0, -1.0)                 # + + - - ...
+    w = np.where(i % 2 == 0, 1.0, -1.0)                        # + - + - ...
+    assert z.sum() == 0 and w.sum() == 0 and (z * w).sum() == 0
+    x = (mu + s * z).astype(np.float32)
+    y = (x.astype(np.float64) - d * w).astype(np.float32)
+    assert np.array_equal(x.astype(np.float64) - y.astype(np.float64), d * w)   # errors exact
+    q = oracle.quality(x, y)
+    assert abs(q["norm_err"] / math.sqrt(n) - d) < 1e-9 * d
+    assert round(q["pearson"], 6) == P_PEARSON, q["pearson"]
+    assert round(q["norm_err_norm"], 6) == P_NORM_ERR_NORM, q["norm_err_norm"]
+    # and the centred reading would have printed a different number
+    xc = x.astype(np.float64) - x.astype(np.float64).mean()
+    assert round(q["norm_err"] / math.sqrt(float((xc * xc).sum())), 6) != P_NORM_ERR_NORM
+
+
+def test_norm_err_norm_closed_forms():
+    """Hand-computed values: x = 4 everywhere, e = +-1/4 -> ||e|| = sqrt(n)/4,
+    ||x|| = 4 sqrt(n), ratio exactly 1/16; x = (3, 4) pairs with e = 1/2 on
+    the 4s only -> ratio = sqrt(n/2 * 1/4) / sqrt(n/2 * 25) = 1/10."""
+    n = 1024
+    x = np.full(n, 4.0, np.float32)
+    y = (x + np.where(np.arange(n) % 2 == 0, 0.25, -0.25)).astype(np.float32)
+    assert oracle.quality(x, y)["norm_err_norm"] == 1 / 16
+    x = np.tile(np.array([3.0, 4.0], np.float32), n // 2)
+    y = x.copy()
+    y[1::2] = 3.5
+    assert abs(oracle.quality(x, y)["norm_err_norm"] - 0.1) < 1e-16
