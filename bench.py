@@ -2,35 +2,42 @@
 """bench.py -- throughput of the cuSZp hot path on B200 (BASELINE.json metric).
 
     python bench.py [--gpus N --steps K --warmup W] [--impl ours|reference]
-                    [--config c2_hurricane|c1_smooth1d|c3_hacc|c4_nyx|c5_rtm]
+                    [--config c3_hacc|c5_rtm|c1_smooth1d|c2_hurricane|c4_nyx]
 
 A STEP is one pass of the whole hot path over one
-batch of synthetic input: for every field of the config and every REL error
-bound it names, value range (a1) -> fused compression (a2..a8) -> fused
-decompression (a9..a12), all through the C ABI.  The default workload is
-BASELINE configs[1]: three Hurricane-shaped 100x500x500 fp32 fields (U,
-QCLOUD, TC) at REL 1e-2, 1e-3, 1e-4 -> 9 round trips, 900 MB of fp32 input
-per step per GPU.
+batch of synthetic input: for every field of the config and every REL bound
+it names, value range (a1) -> fused compression (a2..a8) -> fused
+decompression (a9..a12), all through the C ABI.
 
-Timing: the L2 (126 MB) is flushed (a 512 MB write + read, untimed) before every
-round trip; each round trip is bracketed by CUDA events on the launching
-stream; a step's time is the sum of its round trips' device time.  W warm-up
-steps, then K timed steps between barrier + synchronize; max over ranks.
-Multi-GPU (torchrun): weak scaling -- every rank compresses its own fields
-with the GLOBAL REL range (NCCL all-gather of (min,max)) and all-gathers the
-compressed byte counts to build the container header (paper_conf_sc_
-huangd0lc23_b200.dist).
+Workload (config.workload):
+  N = 1  the largest single-GPU configuration of BASELINE.json, configs[2]:
+         the HACC-shaped 1D field, 280,953,867 fp32 (1.124 GB), REL 1e-3
+         (default --config c3_hacc);
+  N > 1  configs[4]: ONE RTM-shaped 6.82 GB snapshot set (36 x 449x449x235
+         fp32) SHARDED across the N ranks in block-aligned slabs (the
+         north_star split): rank p compresses its slab against the
+         GLOBAL range (NCCL all-gather of 8 B per rank) and the compressed
+         byte counts are all-gathered into the container header (8 B per
+         rank) -- both exchanges inside the timed region (default
+         --config c5_rtm; "scaling": "strong", total work fixed).
+The other configs are reported as secondary keys at N = 1 (c1 as a CUDA-graph
+replay, c2's 9 round trips, c4, and c5 on one GPU).
+
+Timing: the L2 (126 MB) is flushed (a 512 MB write + read, untimed) before
+every round trip; each kernel is bracketed by CUDA events on the launching
+stream; a step's time is the sum of its kernels' device time (max over
+ranks).  W warm-up steps, then K timed steps between barrier + synchronize.
 
 --impl reference runs the CPU oracle (oracle/, single thread) on a bounded
-sample of the same config -- the tier's reference arm.
+sample of the same workload -- the tier's reference arm.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import platform
 import statistics
-import subprocess
 import sys
 import threading
 import time
@@ -45,6 +52,8 @@ import torch  # noqa: E402
 PAPER_A100 = {"compress_mean_gbs": 93.63, "decompress_mean_gbs": 120.04,
               "source": "PAPER.md P:961-962 (A100 40GB, real SDRBench data, REL 1E-1..1E-4)"}
 FALLBACK_HBM_GBS = 6650.0
+METRIC = "end-to-end compress+decompress GB/s (input fp32), REL, incl. range kernel"
+REF_SAMPLE = 1 << 24      # elements per field in each reference step (16 windows of 2^20)
 
 
 def parse_args():
@@ -53,11 +62,12 @@ def parse_args():
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--config", default="c2_hurricane")
+    p.add_argument("--config", default=None, help="default: c3_hacc at N = 1, c5_rtm (sharded) at N > 1")
     p.add_argument("--no-e2e", action="store_true")
-    p.add_argument("--no-large", action="store_true", help="skip the 1.12 GB HACC-shaped context measurement")
+    p.add_argument("--no-secondary", action="store_true", help="skip the c1/c2/c4/c5 secondary keys")
+    p.add_argument("--no-variants", action="store_true", help="skip the block-length / predictor variants")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--cpu-seconds", type=float, default=10.0)
+    p.add_argument("--cpu-seconds", type=float, default=12.0)
     return p.parse_args()
 
 
@@ -73,11 +83,22 @@ def peak_hbm():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def host_info() -> dict:
+    model = platform.processor() or ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
 class ClockSampler:
     """SM clock + clock-event (throttle) reasons polled through NVML every
-    ~2 ms from a thread while the timed region runs (the region lasts tens of
-    ms, too short for nvidia-smi's 100 ms sampling).  Falls back to
-    nvidia-smi when NVML is unavailable."""
+    ~2 ms from a thread while the timed region runs."""
     NAMES = {"hw_slowdown": "nvmlClocksEventReasonHwSlowdown",
              "hw_thermal_slowdown": "nvmlClocksEventReasonHwThermalSlowdown",
              "sw_thermal_slowdown": "nvmlClocksEventReasonSwThermalSlowdown",
@@ -132,35 +153,57 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.sm)}
 
 
-def workload(cfg_name: str):
+def resolve_config(args, world: int) -> str:
+    return args.config or ("c3_hacc" if world == 1 else "c5_rtm")
+
+
+def config_jobs(cfg_name: str):
     import synth
 
     c = synth.CONFIGS[cfg_name]
     fields = c.get("fields", [None])
-    return c, fields, c["rel"]
+    return fields, c["rel"]
+
+
+def make_field(cfg_name: str, field, device):
+    import synth
+
+    return synth.field_for_config(cfg_name, device=device, field=field)
+
+
+def slab(n: int, rank: int, world: int):
+    from paper_conf_sc_huangd0lc23_b200 import dist as czd
+
+    return czd.slab_bounds(n, rank, world)
 
 
 # ---------------------------------------------------------------- reference arm
 
-METRIC = "end-to-end compress+decompress GB/s (input fp32), REL, incl. range kernel"
-REF_SAMPLE = 1 << 20      # elements per field in each reference step
-
-
 def run_reference(args, rank, world):
     """The CPU oracle, as it stands, on a bounded sample of the same workload:
-    every step runs the same round-trip mix as our arm (every field x every
-    REL bound) on the first REF_SAMPLE elements of each field."""
+    every step runs the round trips of our arm's step (every field x every
+    REL bound) on REF_SAMPLE elements of each field, taken as 16 evenly spaced
+    2^20-element windows (block aligned) so sparse and dense parts are both
+    represented (RTM's first snapshots are nearly all zero)."""
     if rank != 0:
         return
     import oracle
-    import synth
 
     oracle.build()
-    c, fields, rels = workload(args.config)
+    cfg = resolve_config(args, world)
+    fields, rels = config_jobs(cfg)
+    gen_dev = "cuda" if torch.cuda.is_available() else "cpu"
     samples = {}
     for f in fields:
-        x = synth.field_for_config(args.config, device="cpu", field=f).numpy()
-        samples[f] = x[: min(x.size, REF_SAMPLE)].copy()
+        x = make_field(cfg, f, gen_dev)
+        n = x.numel()
+        if n <= REF_SAMPLE:
+            samples[f] = x.cpu().numpy()
+        else:
+            w = REF_SAMPLE // 16
+            starts = [((k * (n - w)) // 15) // 32 * 32 for k in range(16)]
+            samples[f] = torch.cat([x[s:s + w] for s in starts]).cpu().numpy()
+        del x
     t_steps = []
     n_step = 0
     for i in range(args.warmup + args.steps):
@@ -177,16 +220,18 @@ def run_reference(args, rank, world):
             t_steps.append(dt)
     tot = sum(t_steps)
     gbs = n_step * 4 * len(t_steps) / tot / 1e9
-    sample = f"first {REF_SAMPLE} elements of each field ({', '.join(f for f in fields if f)}) x REL {rels}"
+    sample = (f"{min(REF_SAMPLE, samples[fields[0]].size)} elements of each field "
+              f"({', '.join(f for f in fields if f) or cfg}; 16 evenly spaced windows) x REL {rels}")
     line = {
         "impl": "reference", "metric": METRIC, "value": gbs,
-        "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": tot / len(t_steps) * 1e3, "higher_is_better": True, "scaling": "weak",
+        "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": tot / len(t_steps) * 1e3, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": args.config, "fields": [f for f in fields if f] or None, "rel": rels,
+        "config": {"workload": cfg, "fields": [f for f in fields if f] or None, "rel": rels,
                    "round_trips_per_step": len(fields) * len(rels), "sample": sample},
         "cpu_baseline": {"value": gbs, "unit": "GB/s", "cores": 1, "kind": "oracle",
-                         "sample": sample + ", single-threaded C++ oracle, all round trips of a step"},
+                         "sample": sample + ", single-threaded C++ oracle, all round trips of a step",
+                         "host": host_info()},
         "e2e": {"value": gbs, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -194,350 +239,475 @@ def run_reference(args, rank, world):
 
 # -------------------------------------------------------------------- our arm
 
-def cpu_baseline(args, cfg_name, fields, rels):
+class Runner:
+    """Device buffers + timing of round trips through the C ABI."""
+
+    def __init__(self, dev, nmax: int, world: int = 1, group=None):
+        import paper_conf_sc_huangd0lc23_b200 as cz
+
+        self.cz = cz
+        self.lib = cz.lib()
+        self.dev = dev
+        self.world = world
+        self.group = group
+        self.stream = torch.cuda.current_stream(dev)
+        self.sp = int(self.stream.cuda_stream)
+        self.ws = cz.Workspace(max(nmax, 1), dev)
+        self.cap = cz.max_compressed_bytes(nmax)
+        self.out = torch.empty(self.cap, dtype=torch.uint8, device=dev)
+        self.out_bytes = torch.zeros(1, dtype=torch.int64, device=dev)
+        self.y = torch.empty(max(nmax, 1), dtype=torch.float32, device=dev)
+        self.mm_local = torch.empty(2, dtype=torch.float32, device=dev)
+        self.mm_all = torch.empty(2 * world, dtype=torch.float32, device=dev)
+        self.sizes_all = torch.empty(world, dtype=torch.int64, device=dev)
+        self.flush_buf = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+        self.sink = torch.empty(1, dtype=torch.int64, device=dev)
+
+    def flush_l2(self):
+        # write then read 512 MB (> 126 MB L2): the L2 ends up holding CLEAN lines
+        # of an unrelated buffer -- a write-only flush would leave ~126 MB of
+        # dirty lines whose write-back gets charged to the next timed kernel
+        self.flush_buf.zero_()
+        self.sink.copy_(self.flush_buf.view(torch.int64).sum())
+
+    def round_trip(self, x, n, rel, ev=None):
+        """range -> (all-gather of (min,max)) -> compress -> (all-gather of
+        sizes) -> decompress, events between the stages."""
+        cz, lib, sp = self.cz, self.lib, self.sp
+        from paper_conf_sc_huangd0lc23_b200 import dist as czd
+
+        if ev is not None:
+            ev[0].record(self.stream)
+        cz.check(lib.cuszp_range(x.data_ptr(), n, self.mm_local.data_ptr(), self.ws.ptr(), self.ws.nbytes, sp),
+                 "range")
+        if self.world > 1:
+            czd.allgather_minmax(self.mm_local, self.mm_all, self.group)   # global REL range (NVLink)
+            mm, pairs = self.mm_all, self.world
+        else:
+            mm, pairs = self.mm_local, 1
+        if ev is not None:
+            ev[1].record(self.stream)
+        cz.check(lib.cuszp_compress_minmax(x.data_ptr(), n, float(rel), mm.data_ptr(), pairs, self.out.data_ptr(),
+                                           self.cap, self.out_bytes.data_ptr(), self.ws.ptr(), self.ws.nbytes, sp),
+                 "compress")
+        if self.world > 1:
+            czd.allgather_sizes(self.out_bytes, self.group, self.sizes_all)   # container header offsets
+        if ev is not None:
+            ev[2].record(self.stream)
+        cz.check(lib.cuszp_decompress(self.out.data_ptr(), self.cap, self.y.data_ptr(), n, self.ws.ptr(),
+                                      self.ws.nbytes, sp), "decompress")
+        if ev is not None:
+            ev[3].record(self.stream)
+
+    def measure(self, jobs, steps: int, warmup: int, clocks: ClockSampler | None = None):
+        """jobs = [(label, x, n, rel)]; per-kernel device seconds summed over
+        the timed steps (max over ranks), compressed sizes per job."""
+        ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in jobs]
+        acc = {"range": 0.0, "compress": 0.0, "decompress": 0.0}
+        sizes = {}
+        for _ in range(max(warmup, 3)):
+            for lab, x, n, rel in jobs:
+                self.flush_l2()
+                self.round_trip(x, n, rel)
+        torch.cuda.synchronize(self.dev)
+        if self.world > 1:
+            torch.distributed.barrier()
+        torch.cuda.synchronize(self.dev)
+        if clocks is not None:
+            clocks.start()
+        t0 = time.perf_counter()
+        for _ in range(steps):
+            for j, (lab, x, n, rel) in enumerate(jobs):
+                self.flush_l2()                                   # L2 flush, untimed
+                self.round_trip(x, n, rel, ev[j])
+                torch.cuda.synchronize(self.dev)
+                e = ev[j]
+                acc["range"] += e[0].elapsed_time(e[1]) / 1e3
+                acc["compress"] += e[1].elapsed_time(e[2]) / 1e3
+                acc["decompress"] += e[2].elapsed_time(e[3]) / 1e3
+                sizes[lab] = int(self.out_bytes.item())
+                assert self.cz.read_header(self.out)["status"] == 0, lab
+        torch.cuda.synchronize(self.dev)
+        wall = time.perf_counter() - t0
+        clk = clocks.stop() if clocks is not None else None
+        if self.world > 1:
+            torch.distributed.barrier()
+        t = torch.tensor([acc["range"], acc["compress"], acc["decompress"]], dtype=torch.float64, device=self.dev)
+        if self.world > 1:
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        acc = dict(zip(("range", "compress", "decompress"), (float(v) for v in t.tolist())))
+        return acc, sizes, wall, clk
+
+
+def summarise(jobs, acc, sizes, steps, world, peak, n_total=None):
+    """Throughputs of a measured job list: GB/s of fp32 input (whole job),
+    per-kernel algorithmic HBM bytes / time and the fraction of the peak."""
+    in_bytes = sum(4 * n for _, _, n, _ in jobs)                  # this rank's input per step
+    # whole-job input: every rank's slab of every job (n_total = elements per step, all ranks)
+    in_total = (4 * n_total if n_total is not None else in_bytes * world) * steps
+    t = acc["range"] + acc["compress"] + acc["decompress"]
+    S = {lab: sizes[lab] for lab, *_ in jobs}
+    alg = {"range": sum(4 * n for _, _, n, _ in jobs),
+           "compress": sum(4 * n + S[lab] for lab, _, n, _ in jobs),
+           "decompress": sum(S[lab] + 4 * n for lab, _, n, _ in jobs)}
+    kernels = {k: {"us_per_step": acc[k] / steps * 1e6,
+                   "algorithmic_gbs": alg[k] * steps / acc[k] / 1e9,
+                   "frac_of_peak": alg[k] * steps / acc[k] / 1e9 / peak} for k in acc}
+    return {
+        "round_trip_gbs": in_total / t / 1e9,
+        "compress_gbs": in_total / (acc["range"] + acc["compress"]) / 1e9,
+        "compress_kernel_only_gbs": in_total / acc["compress"] / 1e9,
+        "decompress_gbs": in_total / acc["decompress"] / 1e9,
+        "rel_compress_frac_of_peak": (alg["range"] + alg["compress"]) * steps / (acc["range"] + acc["compress"])
+        / 1e9 / peak,
+        "cr": {lab: round(4 * n / S[lab], 3) for lab, _, n, _ in jobs},
+        "kernels": kernels,
+        "ms_per_step": t / steps * 1e3,
+        "alg_bytes_per_step": alg,
+    }
+
+
+def cpu_baseline(x_np: np.ndarray, rel: float, seconds: float, label: str) -> dict:
+    """The oracle as it stands on the same field: single-threaded round trips
+    (the baseline proper, cores = 1), plus the same oracle run slab-parallel
+    on every host core (block-aligned slabs against the global range; ctypes
+    releases the GIL) as context."""
+    import concurrent.futures as cf
+
     import oracle
-    import synth
 
     oracle.build()
-    x = synth.field_for_config(cfg_name, device="cpu", field=fields[0]).numpy()
-    rel = rels[len(rels) // 2]
+    n = x_np.size
     n_done, t_tot, reps = 0, 0.0, 0
-    while t_tot < args.cpu_seconds or reps == 0:
+    while t_tot < seconds or reps == 0:
         t0 = time.perf_counter()
-        st, s = oracle.compress(x, rel, oracle.REL)
-        st2, y = oracle.decompress(s, x.size)
+        st, s = oracle.compress(x_np, rel, oracle.REL)
+        st2, y = oracle.decompress(s, n)
         t_tot += time.perf_counter() - t0
-        n_done += x.size
+        assert st == st2 == oracle.OK
+        n_done += n
         reps += 1
+        del s, y
+    hi = host_info()
+    P = max(1, int(hi["nproc"] or 1))
+    lo_, hi_ = oracle.value_range(x_np)
+    mm = np.array([lo_, hi_], np.float32)
+
+    def part(p):
+        s0, s1 = slab(n, p, P)
+        st, s = oracle.compress_minmax(x_np[s0:s1], rel, mm)
+        st2, y = oracle.decompress(s, s1 - s0)
+        return st == st2 == oracle.OK
+
+    t0 = time.perf_counter()
+    oracle.value_range(x_np)
+    with cf.ThreadPoolExecutor(P) as ex:
+        assert all(ex.map(part, range(P)))
+    t_all = time.perf_counter() - t0
     return {"value": n_done * 4 / t_tot / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{reps} round trip(s) of {cfg_name}/{fields[0]} ({x.size} elements) at REL {rel}, "
-                      f"{t_tot:.1f} s single-threaded C++ oracle"}
+            "sample": f"{reps} full round trip(s) of {label} ({n} elements) at REL {rel}: oracle value range + "
+                      f"compress + decompress, {t_tot:.1f} s single-threaded C++ oracle (-O2)",
+            "host": hi,
+            "all_cores": {"value": 4 * n / t_all / 1e9, "unit": "GB/s", "cores": P,
+                          "how": f"the same oracle on {P} block-aligned slabs in {P} threads (global range)"}}
+
+
+def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int) -> dict:
+    """End to end through the asynchronous host-buffer C-ABI calls (pinned
+    memory): every job H2D-copies its field, compresses, moves the stream into
+    host memory (exactly S bytes, SM copy kernel reading the device-side
+    length), brings it back, decompresses and D2H-copies the reconstruction;
+    consecutive jobs rotate over streams so one job's device->host traffic
+    overlaps the next one's host->device traffic.  Wall clock, max over ranks."""
+    n_lanes = int(os.environ.get("CUSZP_E2E_LANES", "2" if nmax > (1 << 27) else "3"))
+    lanes = []
+    for _ in range(n_lanes):
+        lanes.append(dict(stream=torch.cuda.Stream(dev),
+                          h_out=torch.zeros(cap, dtype=torch.uint8).pin_memory(),
+                          h_len=torch.zeros(1, dtype=torch.int64).pin_memory(),
+                          h_y=torch.empty(nmax, dtype=torch.float32).pin_memory(),
+                          d_in=torch.empty(nmax, dtype=torch.float32, device=dev),
+                          d_out=torch.empty(cap, dtype=torch.uint8, device=dev),
+                          d_y=torch.empty(nmax, dtype=torch.float32, device=dev),
+                          ws=cz.Workspace(nmax, dev)))
+    lens = {}
+    k = 0
+    for i in range(1 + steps):
+        if i == 1:
+            torch.cuda.synchronize(dev)
+            if world > 1:
+                torch.distributed.barrier()
+            t0 = time.perf_counter()
+        for lab, h_in, rel in jobs_host:
+            ln = lanes[k % n_lanes]
+            k += 1
+            n = h_in.numel()
+            cz.compress_host_async(h_in, rel, "rel", ln["h_out"], ln["h_len"], ln["d_in"][:n], ln["d_out"],
+                                   ln["ws"], stream=ln["stream"])
+            cz.decompress_host_async(ln["h_out"], ln["h_y"][:n], ln["d_out"], ln["d_y"][:n], ln["ws"],
+                                     stream=ln["stream"])
+            if i == 0:      # warm-up pass: record the stream lengths (bytes counted per step)
+                ln["stream"].synchronize()
+                lens[lab] = int(ln["h_len"].item())
+    torch.cuda.synchronize(dev)
+    t_e2e = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+    if world > 1:
+        torch.distributed.all_reduce(t_e2e, op=torch.distributed.ReduceOp.MAX)
+    h2d = d2h = 0
+    for lab, h_in, rel in jobs_host:
+        n = h_in.numel()
+        h2d += 4 * n + lens[lab]              # field in, stream back in
+        d2h += lens[lab] + 8 + 4 * n          # stream + its length out, reconstruction out
+    # the last job's reconstruction in host memory satisfies the bound
+    lab, h_in, rel = jobs_host[-1]
+    ln = lanes[(k - 1) % n_lanes]
+    n = h_in.numel()
+    eb_l = float(np.frombuffer(ln["h_out"][16:20].numpy().tobytes(), np.float32)[0])
+    err = (ln["h_y"][:n].double() - h_in.double()).abs().max().item()
+    assert err <= eb_l + float(np.spacing(np.float32(h_in.abs().max().item()))), (err, eb_l)
+    del lanes
+    # the host link's own ceiling for this traffic: both directions at once (copy engines)
+    s1, s2 = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+    pa = torch.empty(1 << 28, dtype=torch.uint8).pin_memory()
+    pb = torch.empty(1 << 28, dtype=torch.uint8).pin_memory()
+    da = torch.empty(1 << 28, dtype=torch.uint8, device=dev)
+    db = torch.empty(1 << 28, dtype=torch.uint8, device=dev)
+
+    def both_ways():
+        with torch.cuda.stream(s1):
+            da.copy_(pa, non_blocking=True)
+        with torch.cuda.stream(s2):
+            pb.copy_(db, non_blocking=True)
+
+    both_ways()                                     # first touch of the pinned pages, untimed
+    torch.cuda.synchronize(dev)
+    tl0 = time.perf_counter()
+    for _ in range(4):
+        both_ways()
+    torch.cuda.synchronize(dev)
+    link_gbs = 4 * (1 << 28) / (time.perf_counter() - tl0) / 1e9     # per direction
+    in_step = sum(4 * h.numel() for _, h, _ in jobs_host)
+    bound = in_step / (max(h2d, d2h) / (link_gbs * 1e9)) / 1e9 * world
+    return {"value": in_step * steps * world / float(t_e2e.item()) / 1e9, "unit": "GB/s",
+            "link_gbs_per_direction": round(link_gbs, 1), "link_bound_gbs": round(bound, 1),
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "path": "cuszp_compress_host_async + cuszp_decompress_host_async (pinned host buffers, "
+                    f"{n_lanes} streams, wall clock)"}
+
+
+def graph_replay_c1(r: Runner, steps: int, peak: float) -> dict:
+    """c1 (2^20 elements, launch-bound) as a CUDA-graph replay of range +
+    compress + decompress, L2 flushed before every replay."""
+    x = make_field("c1_smooth1d", None, r.dev)
+    n = x.numel()
+    rel = config_jobs("c1_smooth1d")[1][0]
+    s = torch.cuda.Stream(r.dev)
+    s.wait_stream(torch.cuda.current_stream(r.dev))
+    saved = (r.stream, r.sp)
+    r.stream, r.sp = s, int(s.cuda_stream)
+    with torch.cuda.stream(s):
+        r.round_trip(x, n, rel)                          # library init outside capture
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        r.round_trip(x, n, rel)
+    r.stream, r.sp = saved
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for i in range(3 + steps):
+        r.flush_l2()
+        torch.cuda.synchronize(r.dev)
+        with torch.cuda.stream(s):
+            e0.record(s)
+            g.replay()
+            e1.record(s)
+        torch.cuda.synchronize(r.dev)
+        if i >= 3:
+            ts.append(e0.elapsed_time(e1) / 1e3)
+    assert r.cz.read_header(r.out)["status"] == 0
+    S = int(r.out_bytes.item())
+    t = float(np.median(ts))
+    # eager, same flush protocol, for comparison
+    jobs = [("c1", x, n, rel)]
+    acc, sizes, _, _ = r.measure(jobs, steps, 3)
+    te = (acc["range"] + acc["compress"] + acc["decompress"]) / steps
+    return {"workload": f"c1_smooth1d (2^20 fp32) REL {rel:g}", "cr": round(4 * n / S, 3),
+            "graph_round_trip_us": round(t * 1e6, 2), "graph_round_trip_gbs": round(4 * n / t / 1e9, 1),
+            "eager_round_trip_us": round(te * 1e6, 2), "eager_round_trip_gbs": round(4 * n / te / 1e9, 1),
+            "note": "inputs fit in L2 (4 MB); flushed before every replay"}
+
+
+def secondary(r: Runner, cfg: str, steps: int, peak: float) -> dict:
+    fields, rels = config_jobs(cfg)
+    xs = {f: make_field(cfg, f, r.dev) for f in fields}
+    jobs = [(f"{f}@{rel:g}" if f else f"{rel:g}", xs[f], xs[f].numel(), rel) for f in fields for rel in rels]
+    acc, sizes, _, _ = r.measure(jobs, steps, 3)
+    d = summarise(jobs, acc, sizes, steps, 1, peak)
+    jobs_n = jobs[0][2]
+    del xs, jobs
+    torch.cuda.empty_cache()
+    return {"workload": cfg, "n_per_field": jobs_n, **{k: d[k] for k in (
+        "round_trip_gbs", "compress_gbs", "decompress_gbs", "rel_compress_frac_of_peak", "cr", "kernels")}}
+
+
+def variants(r: Runner, peak: float, steps: int) -> dict:
+    """Block lengths L and the 2-layer predictor (rank 4)
+    on Hurricane U at REL 1e-3, compress and decompress kernels only, eb from
+    a given range (like for like: no range kernel in any of them), L2 flushed."""
+    cz, lib, sp = r.cz, r.lib, r.sp
+    x0 = make_field("c2_hurricane", "U", r.dev)
+    n0 = x0.numel()
+    rel0 = 1e-3
+    cz.check(lib.cuszp_range(x0.data_ptr(), n0, r.mm_local.data_ptr(), r.ws.ptr(), r.ws.nbytes, sp), "range")
+    mm = r.mm_local.cpu().numpy()
+    eb_abs = float(np.float32(np.float32(rel0) * np.float32(mm[1] - mm[0])))
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    out = {"workload": f"c2_hurricane/U@{rel0:g}", "unit": "GB/s of fp32 input"}
+    for Lb, order in ((8, 1), (16, 1), (32, 1), (64, 1), (128, 1), (32, 2)):
+        tc, td = [], []
+        capL = cz.max_compressed_bytes(n0, Lb)
+        outL = r.out if capL <= r.cap else torch.empty(capL, dtype=torch.uint8, device=r.dev)
+        for _ in range(steps + 1):
+            r.flush_l2()
+            ev[0].record(r.stream)
+            if order == 1:
+                cz.check(lib.cuszp_compress_minmax_L(x0.data_ptr(), n0, float(rel0), r.mm_local.data_ptr(), 1, Lb,
+                                                     outL.data_ptr(), capL, r.out_bytes.data_ptr(), r.ws.ptr(),
+                                                     r.ws.nbytes, sp), "compress_L")
+            else:   # the same bound as ABS (the 2-layer path has no given-range entry point)
+                cz.check(lib.cuszp_compress_ex(x0.data_ptr(), n0, eb_abs, cz.ABS, Lb, order, outL.data_ptr(),
+                                               capL, r.out_bytes.data_ptr(), r.ws.ptr(), r.ws.nbytes, sp),
+                         "compress_ex")
+            ev[1].record(r.stream)
+            torch.cuda.synchronize(r.dev)
+            tc.append(ev[0].elapsed_time(ev[1]))
+            r.flush_l2()
+            ev[0].record(r.stream)
+            cz.check(lib.cuszp_decompress_ex(outL.data_ptr(), capL, r.y.data_ptr(), n0, Lb, order, r.ws.ptr(),
+                                             r.ws.nbytes, sp), "decompress_ex")
+            ev[1].record(r.stream)
+            torch.cuda.synchronize(r.dev)
+            td.append(ev[0].elapsed_time(ev[1]))
+        assert cz.last_status(r.ws) == cz.OK
+        SL = int(r.out_bytes.item())
+        tcm, tdm = float(np.median(tc[1:])) / 1e3, float(np.median(td[1:])) / 1e3
+        out[str(Lb) if order == 1 else f"{Lb}_lorenzo2"] = {
+            "cr": round(4 * n0 / SL, 3),
+            "compress_kernel_gbs": round(4 * n0 / tcm / 1e9, 1),
+            "decompress_kernel_gbs": round(4 * n0 / tdm / 1e9, 1),
+            "compress_frac_of_peak": round((4 * n0 + SL) / tcm / 1e9 / peak, 4),
+            "decompress_frac_of_peak": round((4 * n0 + SL) / tdm / 1e9 / peak, 4)}
+        if outL is not r.out:
+            del outL
+    del x0
+    torch.cuda.empty_cache()
+    return out
+
+
+def verify(r: Runner, jobs) -> dict:
+    """Every job's round trip checked on the device with the fused quality
+    kernel (cuszp_quality, untimed): the bound of DESIGN sec 5 and PSNR."""
+    cz = r.cz
+    q = {"psnr": {}, "max_abs_err_over_eb": {}}
+    for lab, x, n, rel in jobs:
+        r.round_trip(x, n, rel)
+        hdr = cz.read_header(r.out)
+        assert hdr["status"] == 0 and cz.last_status(r.ws) == cz.OK
+        qv = cz.quality(x, r.y[:n], bound=float(hdr["eb_abs"]), sync=False).cpu()
+        ulp_max = float(np.spacing(np.float32(max(abs(qv[0].item()), abs(qv[1].item())))))
+        assert qv[3].item() <= hdr["eb_abs"] + ulp_max, (lab, qv[3].item(), hdr["eb_abs"])
+        q["psnr"][lab] = round(qv[7].item(), 3)
+        q["max_abs_err_over_eb"][lab] = round(qv[3].item() / hdr["eb_abs"], 6)
+    return q
 
 
 def run_ours(args, rank, world, dev):
     import paper_conf_sc_huangd0lc23_b200 as cz
-    import synth
-    from paper_conf_sc_huangd0lc23_b200 import dist as czd
 
-    lib = cz.lib()
-    c, fields, rels = workload(args.config)
-    stream = torch.cuda.current_stream(dev)
-    sp = int(stream.cuda_stream)
-
-    # ---- inputs resident in HBM (generated on the device, seeded per rank)
-    xs = {}
-    for f in fields:
-        xs[f] = synth.field_for_config(args.config, device=dev, field=f)
-        if world > 1 and rank > 0:
-            xs[f] = xs[f].roll(rank * 4099)      # distinct data per rank, same statistics
-    n_of = {f: xs[f].numel() for f in fields}
-    nmax = max(n_of.values())
-    ws = cz.Workspace(nmax, dev)
-    cap = cz.max_compressed_bytes(nmax)
-    out = torch.empty(cap, dtype=torch.uint8, device=dev)
-    out_bytes = torch.zeros(1, dtype=torch.int64, device=dev)
-    y = torch.empty(nmax, dtype=torch.float32, device=dev)
-    mm_local = torch.empty(2, dtype=torch.float32, device=dev)
-    mm_all = torch.empty(2 * world, dtype=torch.float32, device=dev)
-    flush_buf = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-    sink = torch.empty(1, dtype=torch.int64, device=dev)
-
-    def flush_l2():
-        # write then read 512 MB (> 126 MB L2): the L2 ends up holding CLEAN lines
-        # of an unrelated buffer -- a write-only flush would leave ~126 MB of
-        # dirty lines whose write-back gets charged to the next timed kernel
-        flush_buf.zero_()
-        sink.copy_(flush_buf.view(torch.int64).sum())
-
-    jobs = [(f, r) for f in fields for r in rels]
+    cfg = resolve_config(args, world)
+    fields, rels = config_jobs(cfg)
     group = torch.distributed.group.WORLD if world > 1 else None
-
-    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in jobs]
-    acc = {"range": 0.0, "compress": 0.0, "decompress": 0.0}
-    sizes = {}
-
-    def one_step(timed: bool):
-        for j, (f, rel) in enumerate(jobs):
-            x = xs[f]
-            n = n_of[f]
-            flush_l2()                                      # L2 flush, untimed
-            e = ev[j]
-            e[0].record(stream)
-            cz.check(lib.cuszp_range(x.data_ptr(), n, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
-            if world > 1:
-                czd.allgather_minmax(mm_local, mm_all, group)   # global REL range over NVLink
-                mm, pairs = mm_all, world
-            else:
-                mm, pairs = mm_local, 1
-            e[1].record(stream)
-            cz.check(lib.cuszp_compress_minmax(x.data_ptr(), n, float(rel), mm.data_ptr(), pairs, out.data_ptr(),
-                                               cap, out_bytes.data_ptr(), ws.ptr(), ws.nbytes, sp), "compress")
-            if world > 1:
-                czd.allgather_sizes(out_bytes, group)          # container header offsets
-            e[2].record(stream)
-            cz.check(lib.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.ptr(), ws.nbytes, sp),
-                     "decompress")
-            e[3].record(stream)
-            if timed:
-                torch.cuda.synchronize(dev)
-                acc["range"] += e[0].elapsed_time(e[1])
-                acc["compress"] += e[1].elapsed_time(e[2])
-                acc["decompress"] += e[2].elapsed_time(e[3])
-                sizes[(f, rel)] = int(out_bytes.item())
-
-    for _ in range(max(args.warmup, 3)):
-        one_step(False)
-    torch.cuda.synchronize(dev)
-    if world > 1:
-        torch.distributed.barrier()
-    torch.cuda.synchronize(dev)
-    clocks = ClockSampler(dev.index)
-    clocks.start()
-    t_wall0 = time.perf_counter()
-    for _ in range(args.steps):
-        one_step(True)
-    torch.cuda.synchronize(dev)
-    t_wall = time.perf_counter() - t_wall0
-    clk = clocks.stop()
-    if world > 1:
-        torch.distributed.barrier()
-
-    # verification of every round trip on the device with the fused quality
-    # kernel (cuszp_quality; untimed): the bound of
-    # DESIGN sec 5, PSNR per job, and the quality kernel's own HBM rate
-    quality = {"psnr": {}, "max_abs_err_over_eb": {}}
-    qev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
-    q_ms = []
-    for f, rel in jobs:
-        x = xs[f]
-        n = n_of[f]
-        cz.check(lib.cuszp_range(x.data_ptr(), n, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
-        cz.check(lib.cuszp_compress_minmax(x.data_ptr(), n, float(rel), mm_local.data_ptr(), 1, out.data_ptr(),
-                                           cap, out_bytes.data_ptr(), ws.ptr(), ws.nbytes, sp), "compress")
-        cz.check(lib.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.ptr(), ws.nbytes, sp), "decompress")
-        hdr = cz.read_header(out)
-        assert hdr["status"] == 0 and cz.last_status(ws) == cz.OK
-        flush_l2()
-        qev[0].record(stream)
-        qraw = cz.quality(x, y[:n], bound=float(hdr["eb_abs"]), sync=False)
-        qev[1].record(stream)
-        torch.cuda.synchronize(dev)
-        q_ms.append(qev[0].elapsed_time(qev[1]))
-        qv = qraw.cpu()
-        ulp_max = float(np.spacing(np.float32(max(abs(qv[0].item()), abs(qv[1].item())))))
-        assert qv[3].item() <= hdr["eb_abs"] + ulp_max, (f, rel, qv[3].item(), hdr["eb_abs"])
-        quality["psnr"][f"{f}@{rel:g}"] = round(qv[7].item(), 3)
-        quality["max_abs_err_over_eb"][f"{f}@{rel:g}"] = round(qv[3].item() / hdr["eb_abs"], 6)
-    q_bytes = sum(8 * n_of[f] for f, _ in jobs)
-    quality["kernel_gbs"] = q_bytes / (sum(q_ms) / 1e3) / 1e9
-
-    # a large field (HACC-shaped, 1.12 GB, REL 1e-3; BASELINE configs[2]) where
-    # launch ramp and drain are amortised: kernel times and roofline fractions
-    # (context for the 100 MB headline fields; inputs >> L2, median of 3)
-    large = None
-    if not args.no_large and world == 1:
-        xl = synth.field_for_config("c3_hacc", device=dev)
-        nl = xl.numel()
-        capl = cz.max_compressed_bytes(nl)
-        wsl = cz.Workspace(nl, dev)
-        outl = torch.empty(capl, dtype=torch.uint8, device=dev)
-        yl = torch.empty(nl, dtype=torch.float32, device=dev)
-        mml = torch.empty(2, dtype=torch.float32, device=dev)
-        tl = {"range": [], "compress": [], "decompress": []}
-        ev4 = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
-        for _ in range(4):
-            ev4[0].record(stream)
-            cz.check(lib.cuszp_range(xl.data_ptr(), nl, mml.data_ptr(), wsl.ptr(), wsl.nbytes, sp), "range")
-            ev4[1].record(stream)
-            cz.check(lib.cuszp_compress_minmax(xl.data_ptr(), nl, 1e-3, mml.data_ptr(), 1, outl.data_ptr(), capl,
-                                               out_bytes.data_ptr(), wsl.ptr(), wsl.nbytes, sp), "compress")
-            ev4[2].record(stream)
-            cz.check(lib.cuszp_decompress(outl.data_ptr(), capl, yl.data_ptr(), nl, wsl.ptr(), wsl.nbytes, sp),
-                     "decompress")
-            ev4[3].record(stream)
-            torch.cuda.synchronize(dev)
-            for k, (e0, e1) in zip(tl, ((0, 1), (1, 2), (2, 3))):
-                tl[k].append(ev4[e0].elapsed_time(ev4[e1]) / 1e3)
-        assert cz.last_status(wsl) == cz.OK
-        Sl = int(out_bytes.item())
-        med = {k: float(np.median(v[1:])) for k, v in tl.items()}
-        bl = {"range": 4 * nl, "compress": 4 * nl + Sl, "decompress": Sl + 4 * nl}
-        large = {"workload": "c3_hacc (280,953,867 fp32, 1.12 GB) REL 1e-3", "cr": round(4 * nl / Sl, 3),
-                 **{k: {"us": round(med[k] * 1e6, 1), "algorithmic_gbs": round(bl[k] / med[k] / 1e9, 1),
-                        "frac_of_peak": round(bl[k] / med[k] / 1e9 / peak_hbm()[0], 4)} for k in med}}
-        del xl, yl, outl, wsl
-        torch.cuda.empty_cache()
-
-    # block-length variants on the first field at the
-    # middle bound: compress and decompress kernels, L2 flushed, median of 5
-    f0, rel0 = fields[0], rels[len(rels) // 2]
-    x0, n0 = xs[f0], n_of[f0]
-    cz.check(lib.cuszp_range(x0.data_ptr(), n0, mm_local.data_ptr(), ws.ptr(), ws.nbytes, sp), "range")
-    variants = {}
-    for Lb, order in ((8, 1), (16, 1), (32, 1), (64, 1), (128, 1), (32, 2)):
-        tc, td = [], []
-        capL = cz.max_compressed_bytes(n0, Lb)
-        outL = out if capL <= cap else torch.empty(capL, dtype=torch.uint8, device=dev)
-        for _ in range(6):
-            flush_l2()
-            qev[0].record(stream)
-            if order == 1:
-                cz.check(lib.cuszp_compress_minmax_L(x0.data_ptr(), n0, float(rel0), mm_local.data_ptr(), 1, Lb,
-                                                     outL.data_ptr(), capL, out_bytes.data_ptr(), ws.ptr(), ws.nbytes,
-                                                     sp), "compress_L")
-            else:   # 2-layer Lorenzo: REL through the range kernel too
-                cz.check(lib.cuszp_compress_ex(x0.data_ptr(), n0, float(rel0), cz.REL, Lb, order, outL.data_ptr(),
-                                               capL, out_bytes.data_ptr(), ws.ptr(), ws.nbytes, sp), "compress_ex")
-            qev[1].record(stream)
-            torch.cuda.synchronize(dev)
-            tc.append(qev[0].elapsed_time(qev[1]))
-            flush_l2()
-            qev[0].record(stream)
-            cz.check(lib.cuszp_decompress_ex(outL.data_ptr(), capL, y.data_ptr(), n0, Lb, order, ws.ptr(),
-                                             ws.nbytes, sp), "decompress_ex")
-            qev[1].record(stream)
-            torch.cuda.synchronize(dev)
-            td.append(qev[0].elapsed_time(qev[1]))
-        assert cz.last_status(ws) == cz.OK
-        SL = int(out_bytes.item())
-        tcm, tdm = float(np.median(tc[1:])) / 1e3, float(np.median(td[1:])) / 1e3
-        variants[str(Lb) if order == 1 else f"{Lb}_lorenzo2"] = {"cr": round(4 * n0 / SL, 3),
-                             "compress_kernel_gbs": round(4 * n0 / tcm / 1e9, 1),
-                             "decompress_kernel_gbs": round(4 * n0 / tdm / 1e9, 1),
-                             "compress_frac_of_peak": round((4 * n0 + SL) / tcm / 1e9 / peak_hbm()[0], 4),
-                             "decompress_frac_of_peak": round((4 * n0 + SL) / tdm / 1e9 / peak_hbm()[0], 4)}
-
-    t_dev = torch.tensor([acc["range"], acc["compress"], acc["decompress"]], dtype=torch.float64, device=dev)
-    if world > 1:
-        torch.distributed.all_reduce(t_dev, op=torch.distributed.ReduceOp.MAX)
-    t_range, t_comp, t_decomp = (float(v) / 1e3 for v in t_dev.tolist())   # seconds over K steps
-    K = args.steps
-    in_bytes_step = sum(4 * n_of[f] for f, _ in jobs)
-    total_bytes = in_bytes_step * K * world
-    t_step_total = t_range + t_comp + t_decomp
-    S = {k: v for k, v in sizes.items()}
-    cr = {f"{f}@{r:g}": round(4 * n_of[f] / S[(f, r)], 3) for f, r in jobs}
-
     peak, peak_src = peak_hbm()
-    per_launch = {
-        "range": sum(4 * n_of[f] for f, _ in jobs) / (t_range / K),
-        "compress": sum(4 * n_of[f] + S[(f, r)] for f, r in jobs) / (t_comp / K),
-        "decompress": sum(S[(f, r)] + 4 * n_of[f] for f, r in jobs) / (t_decomp / K),
-    }
-    times = {"range": t_range, "compress": t_comp, "decompress": t_decomp}
-    dom = max(times, key=times.get)
-    achieved = per_launch[dom] / 1e9
-    traffic = None
+
+    # ---- inputs resident in HBM: this rank's block-aligned slab of every field
+    xs, n_total = {}, 0
+    for f in fields:
+        full = make_field(cfg, f, dev)
+        n_total += full.numel() * len(rels)
+        s0, s1 = slab(full.numel(), rank, world)
+        xs[f] = full[s0:s1].clone() if world > 1 else full
+        del full
+    torch.cuda.empty_cache()
+    jobs = [(f"{f}@{rel:g}" if f else f"{rel:g}", xs[f], xs[f].numel(), rel) for f in fields for rel in rels]
+    nmax = max(x.numel() for x in xs.values())
+    r = Runner(dev, nmax, world, group)
+    clocks = ClockSampler(dev.index)
+    acc, sizes, wall, clk = r.measure(jobs, args.steps, args.warmup, clocks)
+    K = args.steps
+    d = summarise(jobs, acc, sizes, K, world, peak, n_total=n_total)
+    dom = max(acc, key=acc.get)
+    traffic, traffic_src = None, None
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as fh:
-            traffic = json.load(fh).get("dram_bytes_per_launch", {}).get(dom)
+            js = json.load(fh)
+        if js.get("workload") == cfg:
+            traffic = js.get("dram_bytes_per_launch", {}).get(dom)
+            traffic_src = js.get("source")
     except Exception:
         pass
-
+    achieved = d["kernels"][dom]["algorithmic_gbs"]
     line = {
         "metric": METRIC,
-        "value": total_bytes / t_step_total / 1e9 / K * K,
+        "value": d["round_trip_gbs"],
         "unit": "GB/s", "n_gpus": world, "steps": K, "warmup": max(args.warmup, 3),
-        "ms_per_step": t_step_total / K * 1e3, "higher_is_better": True, "scaling": "weak",
+        "ms_per_step": d["ms_per_step"], "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": args.config, "fields": [f for f in fields if f] or None, "rel": rels,
-                   "n_per_field": n_of[fields[0]], "round_trips_per_step": len(jobs),
-                   "parallelism": f"dp{world}" if world > 1 else "single",
-                   "l2": "flushed (512 MB write + read, untimed) before every round trip"},
-        "compress_gbs": in_bytes_step * K * world / (t_range + t_comp) / 1e9,
-        "compress_kernel_only_gbs": in_bytes_step * K * world / t_comp / 1e9,
-        "decompress_gbs": in_bytes_step * K * world / t_decomp / 1e9,
-        "cr": cr,
-        "kernels": {k: {"ms_per_step": times[k] / K * 1e3, "algorithmic_gbs": per_launch[k] / 1e9,
-                        "frac_of_peak": per_launch[k] / 1e9 / peak} for k in times},
+        "config": {"workload": cfg, "fields": [f for f in fields if f] or None, "rel": rels,
+                   "n_elements": n_total // len(rels), "n_per_rank": [x.numel() for x in xs.values()],
+                   "round_trips_per_step": len(jobs),
+                   "parallelism": f"sharded x{world} (block-aligned slabs, global range)" if world > 1 else "single",
+                   "l2": "inputs > L2; flushed anyway (512 MB write + read, untimed) before every round trip"},
+        "compress_gbs": d["compress_gbs"],
+        "compress_kernel_only_gbs": d["compress_kernel_only_gbs"],
+        "decompress_gbs": d["decompress_gbs"],
+        "rel_compress_frac_of_peak": d["rel_compress_frac_of_peak"],
+        "cr": d["cr"],
+        "kernels": d["kernels"],
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src},
+                     "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                     "peak_source": peak_src,
+                     "algorithmic_bytes_per_launch": d["alg_bytes_per_step"][dom] // len(jobs)},
         "gpu_launches": 3 * len(jobs) * K,
-        "block_len_variants": {"workload": f"{f0}@{rel0:g}", "unit": "GB/s of fp32 input", **variants},
-        "large_field": large,
-        "quality": dict(quality, frac_of_peak=quality["kernel_gbs"] / peak,
-                        kernel="cuszp_quality (fused compareData statistics, untimed verification pass)"),
         "clocks": clk,
-        "wall_s_timed_region": t_wall,
+        "wall_s_timed_region": wall,
         "paper_context": PAPER_A100,
     }
+    line["quality"] = verify(r, jobs)
 
-    # ---- e2e through the asynchronous host-buffer C-ABI calls (pinned memory):
-    # every job H2D-copies its field, compresses, moves the stream into host
-    # memory (exactly S bytes, SM copy kernel reading the device-side length),
-    # brings it back, decompresses and D2H-copies the reconstruction; jobs
-    # rotate over three streams so one job's device->host traffic overlaps
-    # the next jobs' host->device traffic on the link.
     if not args.no_e2e:
-        h_in = {f: xs[f].cpu().pin_memory() for f in fields}
-        lanes = []
-        n_lanes = int(os.environ.get("CUSZP_E2E_LANES", "3"))
-        for _ in range(n_lanes):
-            lanes.append(dict(stream=torch.cuda.Stream(dev),
-                              h_out=torch.zeros(cap, dtype=torch.uint8).pin_memory(),
-                              h_len=torch.zeros(1, dtype=torch.int64).pin_memory(),
-                              h_y=torch.empty(nmax, dtype=torch.float32).pin_memory(),
-                              d_in=torch.empty(nmax, dtype=torch.float32, device=dev),
-                              d_out=torch.empty(cap, dtype=torch.uint8, device=dev),
-                              d_y=torch.empty(nmax, dtype=torch.float32, device=dev),
-                              ws=cz.Workspace(nmax, dev)))
-        h2d = d2h = 0
-        lens = {}
-        for i in range(1 + args.steps):
-            if i == 1:
-                torch.cuda.synchronize(dev)
-                if world > 1:
-                    torch.distributed.barrier()
-                t0 = time.perf_counter()
-            for j, (f, rel) in enumerate(jobs):
-                ln = lanes[j % n_lanes]
-                n = n_of[f]
-                cz.compress_host_async(h_in[f], rel, "rel", ln["h_out"], ln["h_len"], ln["d_in"], ln["d_out"],
-                                       ln["ws"], stream=ln["stream"])
-                cz.decompress_host_async(ln["h_out"], ln["h_y"][:n], ln["d_out"], ln["d_y"], ln["ws"],
-                                         stream=ln["stream"])
-                if i == 0:      # warm-up pass: record the stream lengths (bytes counted per step)
-                    ln["stream"].synchronize()
-                    lens[(f, rel)] = int(ln["h_len"].item())
-        torch.cuda.synchronize(dev)
-        t_e2e = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
-        if world > 1:
-            torch.distributed.all_reduce(t_e2e, op=torch.distributed.ReduceOp.MAX)
-        for f, rel in jobs:
-            n = n_of[f]
-            h2d += 4 * n + lens[(f, rel)]              # field in, stream back in
-            d2h += lens[(f, rel)] + 8 + 4 * n          # stream + its length out, reconstruction out
-        # the last job's reconstruction in host memory satisfies the bound
-        f_l, rel_l = jobs[-1]
-        ln = lanes[(len(jobs) - 1) % n_lanes]
-        eb_l = float(np.frombuffer(ln["h_out"][16:20].numpy().tobytes(), np.float32)[0])
-        err = (ln["h_y"][: n_of[f_l]].double() - h_in[f_l].double()).abs().max().item()
-        assert err <= eb_l + float(np.spacing(np.float32(h_in[f_l].abs().max().item()))), (err, eb_l)
-        # the host link's own ceiling for this traffic: both directions at once (copy engines)
-        pa = torch.empty(1 << 28, dtype=torch.uint8).pin_memory()
-        pb = torch.empty(1 << 28, dtype=torch.uint8).pin_memory()
-        da = torch.empty(1 << 28, dtype=torch.uint8, device=dev)
-        db = torch.empty(1 << 28, dtype=torch.uint8, device=dev)
-        def both_ways():
-            with torch.cuda.stream(lanes[0]["stream"]):
-                da.copy_(pa, non_blocking=True)
-            with torch.cuda.stream(lanes[1]["stream"]):
-                pb.copy_(db, non_blocking=True)
-        both_ways()                                     # first touch of the pinned pages, untimed
-        torch.cuda.synchronize(dev)
-        tl0 = time.perf_counter()
-        for _ in range(4):
-            both_ways()
-        torch.cuda.synchronize(dev)
-        link_gbs = 4 * (1 << 28) / (time.perf_counter() - tl0) / 1e9     # per direction
-        e2e_bound = in_bytes_step / (max(h2d, d2h) / (link_gbs * 1e9)) / 1e9 * world
-        line["e2e"] = {"value": in_bytes_step * K * world / float(t_e2e.item()) / 1e9, "unit": "GB/s",
-                       "link_gbs_per_direction": round(link_gbs, 1), "link_bound_gbs": round(e2e_bound, 1),
-                       "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                       "path": "cuszp_compress_host_async + cuszp_decompress_host_async (pinned host buffers, "
-                               f"{n_lanes} streams, wall clock)"}
+        hx = {}
+        h_jobs = [(lab, hx.setdefault(id(x), x.cpu().pin_memory()), rel) for lab, x, _, rel in jobs]
+        line["e2e"] = e2e_measure(cz, dev, h_jobs, K, world, r.cap, nmax)
+        del h_jobs, hx
+
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(args, args.config, fields, rels)
+        lab, x, n, rel = jobs[len(jobs) // 2]
+        line["cpu_baseline"] = cpu_baseline(x.cpu().numpy(), rel, args.cpu_seconds, f"{cfg}/{lab}")
+
+    del xs, jobs, r
+    torch.cuda.empty_cache()
+    if world == 1 and not args.no_secondary:
+        # every other config at N = 1, each with buffers of its own size
+        sec = {"c1_graph": graph_replay_c1(Runner(dev, 1 << 20), max(K, 10), peak)}
+        torch.cuda.empty_cache()
+        for c, nmax_c in (("c2_hurricane", 25_000_000), ("c4_nyx", 512 ** 3), ("c5_rtm", 1_705_544_460)):
+            if c != cfg:
+                sec[c] = secondary(Runner(dev, nmax_c), c, 5 if c != "c5_rtm" else 3, peak)
+                torch.cuda.empty_cache()
+        line["secondary"] = sec
+    if world == 1 and not args.no_variants:
+        line["block_len_variants"] = variants(Runner(dev, 25_000_000), peak, 5)
+        torch.cuda.empty_cache()
     return line
 
 
