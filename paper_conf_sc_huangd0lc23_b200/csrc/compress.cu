@@ -67,7 +67,8 @@ static_assert(kCW == 8 || kCW == 16, "compute warps");
 constexpr int kCThreads = (kFirstCompute + kCW) * 32;
 static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * 32, "ring size");
 
-struct TileMeta {
+struct alignas(16) TileMeta {
+  uint32_t wb[kTileBlocks / 4];    // words of the 4 sub-blocks of every group (bytes), tile order
   uint32_t tile;
   uint32_t agg;                    // words of the tile
   uint16_t cnt[kCW];               // words per compute warp
@@ -120,6 +121,50 @@ __device__ __forceinline__ void quantize_fast2(float xa, float xb, float two_eb,
   asm("mov.b64 {%0, %1}, %2;" : "=r"(ta), "=r"(tb) : "l"(t));
   rmax = fmaxf(rmax, fmaxf(fabsf(r0a), fabsf(r0b)));       // R5 guard on finite values (Inf too)
   resmax = fmaxf(resmax, fmaxf(fabsf(ra), fabsf(rb)));
+}
+
+// M = 1, O = 1 fast path: the same R2 sequence, and the block Lorenzo step
+// done on SCALED floats.  r0 * 2^-149 is the subnormal float whose bits are
+// sign | |r0| (exact for |r0| < 2^23: the subnormal grid is the integer grid
+// scaled by 2^-149), so the difference of two neighbours, computed exactly by
+// one fma, has bits sign(l) | |l| for |l| < 2^23 (always, under the R5 guard)
+// and a rotate left by one gives v = 2|l| + [l < 0] directly.  lane 0 takes
+// r_{-1} = 0 through k = 0 in l = fma(prev, -k, r): prev * -0 + r = r
+// (+0 for r = +0; r0 = t - magic is never -0).  Data failing the guard give
+// garbage v, as on the integer path: such blocks are flagged ERANGE.
+// Returns the two scaled values packed; updates rmax (|r0|) and resmax.
+__device__ __forceinline__ uint64_t quantize_scaled2(float xa, float xb, float two_eb, float recip, float& rmax,
+                                                     float& resmax) {
+  uint64_t x, t, r0, res, rs;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(x) : "f"(xa), "f"(xb));
+  const uint64_t rc = (uint64_t(__float_as_uint(recip)) << 32) | __float_as_uint(recip);
+  const uint64_t mg = (uint64_t(__float_as_uint(kRoundMagic)) << 32) | __float_as_uint(kRoundMagic);
+  const uint64_t nt = (uint64_t(__float_as_uint(-two_eb)) << 32) | __float_as_uint(-two_eb);
+  const uint64_t sc = 0x0000000100000001ull;                  // 2^-149, the smallest subnormal, twice
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(t) : "l"(x), "l"(rc), "l"(mg));
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r0) : "l"(t), "l"(mg));
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(res) : "l"(r0), "l"(nt), "l"(x));
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(rs) : "l"(r0), "l"(sc));
+  float r0a, r0b, ra, rb;
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(r0a), "=f"(r0b) : "l"(r0));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(ra), "=f"(rb) : "l"(res));
+  rmax = fmaxf(rmax, fmaxf(fabsf(r0a), fabsf(r0b)));       // R5 guard on finite values (Inf too)
+  resmax = fmaxf(resmax, fmaxf(fabsf(ra), fabsf(rb)));
+  return rs;
+}
+
+// v for two rows at once: lanes j take the scaled r_{j-1} (lane 0: k = 0)
+__device__ __forceinline__ void lorenzo_scaled2(uint64_t rs, uint64_t nk, uint32_t& va, uint32_t& vb) {
+  uint32_t a, b;
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(a), "=r"(b) : "l"(rs));
+  const uint32_t pa = __shfl_up_sync(kFull, a, 1), pb = __shfl_up_sync(kFull, b, 1);
+  uint64_t p, l;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(p) : "r"(pa), "r"(pb));
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(l) : "l"(p), "l"(nk), "l"(rs));   // exact: r_j - r_{j-1}
+  uint32_t la, lb;
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(la), "=r"(lb) : "l"(l));
+  va = __funnelshift_l(la, la, 1);                             // sign | |l|  ->  2|l| + sign
+  vb = __funnelshift_l(lb, lb, 1);
 }
 
 __device__ __forceinline__ uint32_t quantize_exact(float x, float eb, float two_eb, float recip, float& rmax) {
@@ -231,6 +276,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           // ticket taken only once the stage is free: a prefetched ticket would
           // wait a whole tile of compute before its load, and every later tile's
           // look-back would wait for it
+          stress_delay(i);
           const uint32_t t = atomicAdd(&a.ws->ticket, 1u);
           if (t >= a.num_tiles) {
             sm.in_tile[s] = kSentinel;
@@ -281,6 +327,20 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const TileMeta& md = sm.meta[m];
         const uint32_t agg = md.agg;
         if (lane == 0 && t > 0) publish_prefix(a.status, t, excl + agg, epoch);
+        {
+          // F bytes of the tile (Fig 12 part 1): lane L converts group L's word
+          // counts, F = words - 1 (0 for a zero block) bytewise (counts <= 32, no
+          // carries); the stores also cover the F area's zero padding up to
+          // align16(nb) (sub-blocks past n encode as zero blocks, F = 0)
+          const uint32_t wb = md.wb[lane];
+          uint32_t f = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
+          const uint64_t blk = (uint64_t(t) * kTileBlocks + 4u * lane) / M;
+          if (blk < align16(a.nb)) {
+            if constexpr (M == 1) *reinterpret_cast<uint32_t*>(a.out + kHdr + blk) = f;
+            else if constexpr (M == 2) *reinterpret_cast<uint16_t*>(a.out + kHdr + blk) = uint16_t(__byte_perm(f, 0, 0x4420u));
+            else a.out[kHdr + blk] = uint8_t(f);
+          }
+        }
         const uint32_t cnt = lane < kCW ? md.cnt[lane] : 0u;
         const uint32_t hd = lane < kCW ? md.head[lane] : 0u;
         uint32_t incl = cnt;
@@ -297,17 +357,28 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           trace_put(a.trace, t, 6, ns);
         }
 #endif
-        // a8 store: each compute warp's ring segment -> [excl + warp offset, ...)
+        // a8 store: each compute warp's ring segment -> [excl + warp offset, ...):
+        // the segment is at most two linear pieces of the ring (before and
+        // after its wrap point), each copied with running pointers
+        uint32_t* dst_t = payload + excl + lane;
 #pragma unroll 1
         for (int w = 0; w < kCW; ++w) {
           const uint32_t c = __shfl_sync(kFull, cnt, w);
           const uint32_t h = __shfl_sync(kFull, hd, w);
           const uint32_t off = __shfl_sync(kFull, incl - cnt, w);
-          uint32_t* dst = payload + excl + off;
-          const uint32_t* src = sm.ring[w];
-          for (uint32_t k = lane; k < c; k += 32) dst[k] = src[(h + k) & (kRing - 1)];
+          const uint32_t first = min(c, kRing - h);               // words before the wrap
+          uint32_t* dst = dst_t + off;
+          const uint32_t* src = sm.ring[w] + h + lane;
+#pragma unroll 4
+          for (int k = lane; k < int(first); k += 32, src += 32, dst += 32) *dst = *src;
+          src = sm.ring[w] + lane;
+          dst = dst_t + off + first;
+#pragma unroll 2
+          for (int k = lane; k < int(c - first); k += 32, src += 32, dst += 32) *dst = *src;
         }
         // release ring space in CTA tile order
+        if (lane == 0) stress_delay(j ^ 0x55u);
+        __syncwarp();
         while (ld_volatile_u32(&sm.released) != j) __nanosleep(64);
         if (lane < kCW) sm.tail[lane] += cnt;
         __syncwarp();
@@ -321,6 +392,10 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       // ------------------------------------------------------------ compute
       const int w = warp - kFirstCompute;
       const Xpose xpose(lane);
+      // scaled-float Lorenzo (quantize_scaled2) for the paper's default L = 32, order 1
+      constexpr bool kScaled = (M == 1 && O == 1);
+      const float kf = lane ? -1.0f : -0.0f;
+      const uint64_t nk = (uint64_t(__float_as_uint(kf)) << 32) | __float_as_uint(kf);
       uint32_t head = 0;                                // words this warp has appended (monotonic)
       uint32_t* ring = sm.ring[w];
       for (uint32_t i = 0;; ++i) {
@@ -340,11 +415,23 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         if (t != kSentinel && w == 0 && lane == 0) trace_put(a.trace, t, 1, global_ns());
 #endif
         if (t == kSentinel) break;                    // the writers stop on the ticket ring
-        const bool last = (t == a.num_tiles - 1);
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kCBPW * 32;   // first element of the warp
-        const float* src = &sm.in[s][w * kCBPW * 32];
+        float* src = &sm.in[s][w * kCBPW * 32];
+        if (t == a.num_tiles - 1) {
+          // virtual zero pad (R8): the ragged part of the last tile is zeroed in
+          // shared memory once, so the encode loop needs no per-element test.
+          // (No TMA writes this stage again in this launch: the producer's next
+          // ticket is a sentinel; the proxy fence orders it anyway.)
+          for (int k = lane; k < kCBPW * 32; k += 32)
+            if (g0 + k >= a.n) src[k] = 0.0f;
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          __syncwarp();
+        }
         uint32_t cursor = 0;
-        uint32_t fpack[kCBPW / 4];
+        // free words in this warp's ring (refreshed only when a worst-case
+        // group would not fit)
+        uint32_t room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
+        uint32_t wbs[kCBPW / 4];                       // word counts of each group (bytes), for the F array
         // Groups of 4 blocks.  The bit transpose packs as many blocks as fit
         // in 32 bits: 4 blocks when every v < 2^8 (F <= 7), 2 when v < 2^16,
         // else 1.  After it, lane q*W + k holds word k of block q (W = 32 /
@@ -360,12 +447,17 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
             x[q] = src[(4 * g + q) * 32 + lane];
-            if (last && g0 + (4 * g + q) * 32 + lane >= a.n) x[q] = 0.0f;   // virtual zero pad (R8)
           }
           uint32_t r[4];
           float resmax = 0.0f;
-          quantize_fast2(x[0], x[1], two_eb, recip, vmax, resmax, r[0], r[1]);
-          quantize_fast2(x[2], x[3], two_eb, recip, vmax, resmax, r[2], r[3]);
+          uint64_t rs01 = 0, rs23 = 0;
+          if constexpr (kScaled) {
+            rs01 = quantize_scaled2(x[0], x[1], two_eb, recip, vmax, resmax);
+            rs23 = quantize_scaled2(x[2], x[3], two_eb, recip, vmax, resmax);
+          } else {
+            quantize_fast2(x[0], x[1], two_eb, recip, vmax, resmax, r[0], r[1]);
+            quantize_fast2(x[2], x[3], two_eb, recip, vmax, resmax, r[2], r[3]);
+          }
           // NaN residuals are not caught here (fmax drops NaN) but NaN/Inf data
           // always yield a block with > 25 words below (flagged, R5)
 #ifdef CUSZP_C_EAGER_RARE
@@ -381,6 +473,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           const bool rare = __any_sync(kFull, resmax > eb);
 #endif
           uint32_t v[4], wq[4];
+          auto counts = [&]() {
+            // a5: words per block = bit length of the block's OR of v (= of its max)
+#pragma unroll
+            for (int q = 0; q < 4; ++q) wq[q] = 32u - __clz(__reduce_or_sync(kFull, v[q]));
+          };
           auto lorenzo_and_counts = [&]() {
             if constexpr (M == 1) {
 #pragma unroll
@@ -396,15 +493,15 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #ifdef CUSZP_DIAG_TINY
             v[0] = v[1] = v[2] = v[3] = 0;   // diagnostics only: all zero blocks (wrong output)
 #endif
-            // a5: words per block = bit length of the block's OR of v (= of its max)
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              uint32_t b;
-              asm("bfind.u32 %0, %1;" : "=r"(b) : "r"(__reduce_or_sync(kFull, v[q])));   // -1 for 0
-              wq[q] = b + 1;
-            }
+            counts();
           };
-          lorenzo_and_counts();
+          if constexpr (kScaled) {
+            lorenzo_scaled2(rs01, nk, v[0], v[1]);
+            lorenzo_scaled2(rs23, nk, v[2], v[3]);
+            counts();
+          } else {
+            lorenzo_and_counts();
+          }
 #ifndef CUSZP_C_EAGER_RARE
           if (rare) {
 #pragma unroll
@@ -413,8 +510,10 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           }
 #endif
           // room in this warp's ring for a worst-case group (4 x 32 words)
-          while (head + cursor + 4 * 32 - ld_volatile_u32(&sm.tail[w]) > kRing)
-            __nanosleep(CUSZP_C_POLL_NS);
+          while (cursor + 4 * 32 > room) {
+            room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
+            if (cursor + 4 * 32 > room) __nanosleep(CUSZP_C_POLL_NS);
+          }
           if constexpr (M == 2) {                                        // one F per block
             wq[0] = wq[1] = max(wq[0], wq[1]);
             wq[2] = wq[3] = max(wq[2], wq[3]);
@@ -474,39 +573,22 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             }
           }
           cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
-          // F = words - 1 (0 for a zero block), bytewise (counts <= 32, no carries)
-          fpack[g] = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
-          if constexpr (M == 2) fpack[g] = __byte_perm(fpack[g], 0, 0x4420u);   // blocks (0,1), (2,3)
-          if constexpr (M == 4) fpack[g] &= 0xffu;                             // one block
-        }
-        // F bytes of the warp's kCBPW / M blocks (Fig 12 part 1): one store;
-        // the stores also cover the F area's zero padding up to align16(nb)
-        // (padding sub-blocks past n encode as zero blocks, F = 0)
-        const uint64_t blk0 = (uint64_t(t) * kTileBlocks + uint64_t(w) * kCBPW) / M;
-        if (lane == 0 && blk0 < align16(a.nb)) {
-          uint32_t fw[4] = {0, 0, 0, 0};                  // the F bytes, little-endian
-#pragma unroll
-          for (int g = 0; g < kCBPW / 4; ++g) {
-            constexpr int kBytes = 4 / M;                   // F bytes per group
-            const int bit = g * kBytes * 8;
-            fw[bit / 32] |= fpack[g] << (bit % 32);
-          }
-          constexpr int kFBytes = kCBPW / M;
-          if constexpr (kFBytes == 16) *reinterpret_cast<uint4*>(a.out + kHdr + blk0) = make_uint4(fw[0], fw[1], fw[2], fw[3]);
-          else if constexpr (kFBytes == 8) *reinterpret_cast<uint2*>(a.out + kHdr + blk0) = make_uint2(fw[0], fw[1]);
-          else if constexpr (kFBytes == 4) *reinterpret_cast<uint32_t*>(a.out + kHdr + blk0) = fw[0];
-          else *reinterpret_cast<uint16_t*>(a.out + kHdr + blk0) = uint16_t(fw[0]);
+          wbs[g] = wb;
         }
         __syncwarp();
         if (lane == 0) {
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
           TileMeta& md = sm.meta[m];
+          // the group word counts go to the writer, which stores the tile's F bytes
+          if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);
+          else *reinterpret_cast<uint2*>(&md.wb[w * 2]) = make_uint2(wbs[0], wbs[1]);
           md.cnt[w] = uint16_t(cursor);
           md.head[w] = uint16_t(head & (kRing - 1));
-          __threadfence_block();
-          if (atomicAdd(&sm.meta_done[m], 1u) == kCW - 1) {
+          uint32_t done;                                   // release: cnt/head before the count; acquire: the others'
+          asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
+                       : "=r"(done) : "r"(smem_u32(&sm.meta_done[m])) : "memory");
+          if (done == kCW - 1) {
             // last warp of the tile: aggregate -> publish at once (look-back, part 1)
-            __threadfence_block();
             uint32_t agg = 0;
 #pragma unroll
             for (int k = 0; k < kCW; ++k)

@@ -66,6 +66,9 @@ bool eb_is_normal(float eb) {
 // Diagnostics: a device buffer of 8 u64 per tile filled by the next launches
 // (tools/trace_scan.py).  Not part of include/cuszp.h; nullptr in production.
 uint64_t* g_trace = nullptr;
+// Diagnostics: persistent grid sizes forced by cuszp_debug_set_grid (0 = the
+// occupancy-derived default); used by the look-back stress tests.
+int g_grid_compress = 0, g_grid_decompress = 0;
 
 uint32_t status_capacity(size_t ws_bytes) {
   const uint64_t c = (ws_bytes - kWsCtrlBytes) / 8;
@@ -99,6 +102,7 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   if (small_L(L)) return compress_small_launch(L, a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
   const int occ = di.occ_c[mi(M)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
+  if (g_grid_compress > 0) grid = uint64_t(g_grid_compress);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   return compress_launch(M, order, unsigned(grid), a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
@@ -269,6 +273,7 @@ int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t 
                                                                                                 : CUSZP_ECUDA;
   const int occ = di.occ_d[mi(M)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
+  if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -422,6 +427,10 @@ int cuszp_version(void) { return CUSZP_VERSION * 100 + 1; }
 
 // diagnostics only (not declared in include/cuszp.h)
 void cuszp_debug_set_trace(void* d_trace) { g_trace = static_cast<uint64_t*>(d_trace); }
+void cuszp_debug_set_grid(int compress_grid, int decompress_grid) {
+  g_grid_compress = compress_grid;
+  g_grid_decompress = decompress_grid;
+}
 int cuszp_debug_occupancy(int* out4) {
   DeviceInfo di;
   if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;

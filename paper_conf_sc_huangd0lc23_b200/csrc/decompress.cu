@@ -81,7 +81,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
   extern __shared__ __align__(128) unsigned char smem_raw[];
   DecompressSmem& sm = *reinterpret_cast<DecompressSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
-  const int warp = threadIdx.x >> 5;
+  const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);   // provably warp-uniform (no divergence checks before warp-sync ops)
   pdl_wait();                                     // compression / previous call complete
   const uint32_t epoch = running_epoch(a.ws);
 
@@ -128,7 +128,10 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
         if (i >= 2) named_sync(kBarFree0 + b, 64);
         ChunkDesc& cd = sm.chunk[b];
         uint32_t c = 0;
-        if (lane == 0) c = atomicAdd(&a.ws->ticket, 1u);
+        if (lane == 0) {
+          stress_delay(i);
+          c = atomicAdd(&a.ws->ticket, 1u);
+        }
         c = __shfl_sync(kFull, c, 0);
         if (c >= num_chunks) {
           if (lane == 0) cd.chunk = kSentinel;
@@ -274,6 +277,12 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
       // ------------------------------------------------------------ compute
       const int w = warp - kDFirstCompute;
       const Xpose xpose(lane);
+      // scaled-float inverse Lorenzo (order 1, any L): 2eb * 2^23 must be finite,
+      // else (2eb >= 2^105, absurd bounds) the integer path runs
+      const float two_eb_s = __fmul_rn(two_eb, 0x1p23f);
+      const bool scaled_ok = isfinite(two_eb_s);
+      const uint64_t two_eb_s2 = (uint64_t(__float_as_uint(two_eb_s)) << 32) | __float_as_uint(two_eb_s);
+      constexpr uint64_t kUp126x2 = 0x7E8000007E800000ull;          // 2^126, twice
       uint32_t* scratch = sm.scratch[w];
       // per-lane constants: quad mode -> block q = lane/8 owns lanes 8q..8q+7;
       // pair mode -> blocks (0,1) in lanes 0-15 / 16-31 of row 0, (2,3) of row 1
@@ -354,6 +363,60 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           }
           __syncwarp();
           const uint4 raw = *reinterpret_cast<const uint4*>(&scratch[row + lane4]);
+          constexpr int kSeg = (32 - 8 * M) << 8;                     // segment = the block's 8 M lanes
+          if (O == 1 && scaled_ok) {
+            // v = 2|l| + s rotated right by one is sign | |l|: the bits of the
+            // subnormal float l * 2^-149 (the encoder's
+            // quantize_scaled2 in reverse).  Every sum the inverse Lorenzo
+            // forms is r_b - r_a of one block, |.| < 2^23 under the R5
+            // guard, so it stays on the subnormal grid and every add is
+            // exact integer arithmetic.
+            float f0 = __uint_as_float(__funnelshift_r(__byte_perm(raw.x, 0, sel), __byte_perm(raw.x, 0, sel), 1));
+            float f1 = __uint_as_float(__funnelshift_r(__byte_perm(raw.y, 0, sel), __byte_perm(raw.y, 0, sel), 1));
+            float f2 = __uint_as_float(__funnelshift_r(__byte_perm(raw.z, 0, sel), __byte_perm(raw.z, 0, sel), 1));
+            float f3 = __uint_as_float(__funnelshift_r(__byte_perm(raw.w, 0, sel), __byte_perm(raw.w, 0, sel), 1));
+            // a11: r_j = sum_{i <= j} l_i within the block
+            f1 = __fadd_rn(f1, f0);
+            f2 = __fadd_rn(f2, f1);
+            f3 = __fadd_rn(f3, f2);
+            float incl = f3;
+            incl = scan_step_up_f(incl, 1, kSeg);
+            incl = scan_step_up_f(incl, 2, kSeg);
+            incl = scan_step_up_f(incl, 4, kSeg);
+            if constexpr (M >= 2) incl = scan_step_up_f(incl, 8, kSeg);
+            if constexpr (M >= 4) incl = scan_step_up_f(incl, 16, kSeg);
+            const float carry = __fsub_rn(incl, f3);                  // exact (same grid)
+            // a12: d' = r * 2eb = (r 2^-149 * 2^126) * (2eb * 2^23): the first
+            // product is exact (r 2^-23, a normal number), so the second is
+            // the single rounding of r * 2eb -- bit-identical to R13.  Pairs
+            // on the packed fp32 pipe (same RN semantics per element).
+            uint64_t p01, p23, d01, d23;
+            asm("mov.b64 %0, {%1, %2};" : "=l"(p01) : "f"(f0), "f"(f1));
+            asm("mov.b64 %0, {%1, %2};" : "=l"(p23) : "f"(__fadd_rn(f2, carry)), "f"(incl));
+            const uint64_t cc = (uint64_t(__float_as_uint(carry)) << 32) | __float_as_uint(carry);
+            asm("add.rn.f32x2 %0, %0, %1;" : "+l"(p01) : "l"(cc));
+            asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d01) : "l"(p01), "l"(kUp126x2));
+            asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d23) : "l"(p23), "l"(kUp126x2));
+            asm("mul.rn.f32x2 %0, %0, %1;" : "+l"(d01) : "l"(two_eb_s2));
+            asm("mul.rn.f32x2 %0, %0, %1;" : "+l"(d23) : "l"(two_eb_s2));
+            float4 d;
+            asm("mov.b64 {%0, %1}, %2;" : "=f"(d.x), "=f"(d.y) : "l"(d01));
+            asm("mov.b64 {%0, %1}, %2;" : "=f"(d.z), "=f"(d.w) : "l"(d23));
+            float* o = outp + g * 128;
+            if (!last) {
+              *reinterpret_cast<float4*>(o) = d;
+            } else {
+              const uint64_t i0 = uint64_t(o - a.out);
+              if (i0 + 4 <= a.n) *reinterpret_cast<float4*>(o) = d;
+              else {
+                if (i0 < a.n) o[0] = d.x;
+                if (i0 + 1 < a.n) o[1] = d.y;
+                if (i0 + 2 < a.n) o[2] = d.z;
+              }
+            }
+            __syncwarp();
+            continue;
+          }
           // sign-magnitude v = 2|l| + s -> l
           int e0, e1, e2, e3;
           {
@@ -369,7 +432,6 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           e2 += e1;
           e3 += e2;
           int incl = e3;
-          constexpr int kSeg = (32 - 8 * M) << 8;                     // segment = the block's 8 M lanes
           incl = scan_step_up(incl, 1, kSeg);
           incl = scan_step_up(incl, 2, kSeg);
           incl = scan_step_up(incl, 4, kSeg);

@@ -223,6 +223,23 @@ __device__ __forceinline__ void trace_put(uint64_t* trace, uint32_t t, int slot,
   if (trace) trace[8ull * t + slot] = v;
 }
 
+// Look-back stress build (-DCUSZP_STRESS, tests/test_gpu_stress.py): a
+// pseudo-random delay (1 call in 4, up to ~4 us) before every status-word
+// publication, ticket and ring release, so predecessors publish out of order
+// and late, exercising every path of the look-back and of the ring
+// bookkeeping.  Compiled out of the production library.
+#ifdef CUSZP_STRESS
+__device__ __forceinline__ void stress_delay(uint32_t salt) {
+  uint32_t h = salt * 0x9E3779B1u ^ uint32_t(global_ns()) ^ (blockIdx.x * 0x85EBCA6Bu);
+  h ^= h >> 15;
+  h *= 0x2C1B3C6Du;
+  h ^= h >> 12;
+  if ((h & 3u) == 0) __nanosleep(h >> 20);
+}
+#else
+__device__ __forceinline__ void stress_delay(uint32_t) {}
+#endif
+
 // ------------------------------------------------------------- warp helpers
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
@@ -246,6 +263,7 @@ __device__ __forceinline__ uint32_t running_epoch(const WsCtrl* ws) {
 __device__ __forceinline__ void publish_aggregate(uint64_t* status, uint32_t t, uint64_t agg,
                                                   uint32_t epoch) {
   const uint64_t tag = uint64_t(epoch) << kEpochShift;
+  stress_delay(t * 2u);
   st_relaxed_u64(status + t, tag | (t == 0 ? kPrefixFlag : 0ull) | agg);
 }
 
@@ -316,6 +334,7 @@ __device__ __forceinline__ uint64_t resolve_excl(const uint64_t* status, uint32_
 
 // publish_prefix: one thread; tile t's inclusive prefix.
 __device__ __forceinline__ void publish_prefix(uint64_t* status, uint32_t t, uint64_t incl, uint32_t epoch) {
+  stress_delay(t * 2u + 1u);
   st_relaxed_u64(status + t, (uint64_t(epoch) << kEpochShift) | kPrefixFlag | incl);
 }
 
@@ -337,6 +356,18 @@ __device__ __forceinline__ int scan_step_up(int x, int o, int seg_c) {
       " shfl.sync.up.b32 t|p, %0, %1, %2, 0xffffffff;\n"
       " @p add.s32 %0, %0, t;\n}"
       : "+r"(x)
+      : "r"(o), "r"(seg_c));
+  return x;
+}
+
+// The same step on subnormal-scaled floats (decompress, order 1): exact as
+// long as every partial sum stays on the subnormal grid.
+__device__ __forceinline__ float scan_step_up_f(float x, int o, int seg_c) {
+  asm volatile(
+      "{\n .reg .pred p;\n .reg .b32 t;\n"
+      " shfl.sync.up.b32 t|p, %0, %1, %2, 0xffffffff;\n"
+      " @p add.rn.f32 %0, %0, t;\n}"
+      : "+f"(x)
       : "r"(o), "r"(seg_c));
   return x;
 }
