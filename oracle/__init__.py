@@ -71,6 +71,15 @@ def lib():
             h.oracle_decompress.argtypes = [vp, u64, vp, u64]
             h.oracle_decompress.restype = i32
             h.oracle_quality.argtypes = [vp, vp, u64, C.c_double, vp, vp]
+            h.oracle_num_blocks_md.argtypes = [u64, u64, u64, i32]
+            h.oracle_num_blocks_md.restype = u64
+            h.oracle_max_compressed_bytes_md.argtypes = [u64, u64, u64, i32]
+            h.oracle_max_compressed_bytes_md.restype = u64
+            h.oracle_block_lorenzo_md.argtypes = [vp, i32, vp]
+            h.oracle_compress_md.argtypes = [vp, u64, u64, u64, i32, f32, i32, vp, u64, vp]
+            h.oracle_compress_md.restype = i32
+            h.oracle_decompress_md.argtypes = [vp, u64, vp, u64, u64, u64, i32]
+            h.oracle_decompress_md.restype = i32
             h.oracle_block_lorenzo_L.argtypes = [vp, C.c_size_t, i32, vp]
             h.oracle_encode_block_L.argtypes = [vp, i32, vp]
             h.oracle_encode_block_L.restype = i32
@@ -240,6 +249,49 @@ def compress_minmax_L(x, lam: float, minmax, Lb: int) -> tuple[int, np.ndarray]:
     st = lib().oracle_compress_minmax_L(_ptr(x), x.size, np.float32(lam), _ptr(mm), mm.size // 2, int(Lb), _ptr(out),
                                         cap, _ptr(nbytes))
     return st, out[: int(nbytes[0])].copy() if st in (OK, ERANGE) else out[:0]
+
+
+# ---- multi-dimensional Lorenzo (DESIGN R18)
+
+def num_blocks_md(shape, dims: int) -> int:
+    nz, ny, nx = _shape3(shape)
+    return int(lib().oracle_num_blocks_md(nz, ny, nx, int(dims)))
+
+
+def _shape3(shape):
+    shape = tuple(int(v) for v in shape)
+    return (1,) * (3 - len(shape)) + shape
+
+
+def block_lorenzo_md(r, dims: int) -> np.ndarray:
+    """Block-local Lorenzo of ONE block (32 integers in block order)."""
+    r = np.ascontiguousarray(r, dtype=np.int32)
+    assert r.size == 32
+    out = np.zeros(32, np.int32)
+    lib().oracle_block_lorenzo_md(_ptr(r), int(dims), _ptr(out))
+    return out
+
+
+def compress_md(x, shape, dims: int, eb: float, mode: int = REL) -> tuple[int, np.ndarray]:
+    """x: the field (any array of prod(shape) float32, C order), shape
+    (ny, nx) or (nz, ny, nx); dims 2 or 3."""
+    x = _f32(x).ravel()
+    nz, ny, nx = _shape3(shape)
+    assert x.size == nz * ny * nx
+    cap = int(lib().oracle_max_compressed_bytes_md(nz, ny, nx, int(dims)))
+    out = np.zeros(cap, np.uint8)
+    nbytes = np.zeros(1, np.uint64)
+    st = lib().oracle_compress_md(_ptr(x), nz, ny, nx, int(dims), np.float32(eb), int(mode), _ptr(out), cap,
+                                  _ptr(nbytes))
+    return st, out[: int(nbytes[0])].copy() if st in (OK, ERANGE) else out[:0]
+
+
+def decompress_md(stream, shape, dims: int) -> tuple[int, np.ndarray]:
+    s = np.ascontiguousarray(stream, dtype=np.uint8)
+    nz, ny, nx = _shape3(shape)
+    out = np.zeros(nz * ny * nx, np.float32)
+    st = lib().oracle_decompress_md(_ptr(s), s.size, _ptr(out), nz, ny, nx, int(dims))
+    return st, out
 
 
 QUALITY_KEYS = ("min", "max", "range", "max_abs_err", "max_rel_err", "max_pw_rel_err", "mse", "psnr", "nrmse",

@@ -65,6 +65,8 @@ void write_header(uint8_t* out, uint64_t n, int mode, int status, float eb_abs,
   put_u64(out + 24, payload_bytes);
 }
 
+uint64_t encode_and_place(const int32_t* l, uint64_t nb, int L, uint8_t* out);
+
 /* Compression of x[0..n) with a resolved absolute bound eb_abs (sec 3.1,
  * Fig 2): Quantisation and Prediction -> Fixed-length Encoding ->
  * Global Synchronization -> Block Bit-shuffle. */
@@ -98,6 +100,16 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
   std::vector<int32_t> l(static_cast<size_t>(nb * L));
   block_lorenzo_order(r.data(), size_t(nb), L, order, l.data());
 
+  const uint64_t payload_bytes = encode_and_place(l.data(), nb, L, out);
+  write_header(out, n, mode, ORACLE_OK, eb_abs, eb_in, payload_bytes, L);
+  *out_bytes = HEADER_BYTES + align16(nb) + payload_bytes;
+  return ORACLE_OK;
+}
+
+/* Steps (2)-(4) of compression for nb blocks of Lorenzo integers l[nb*L]:
+ * the F bytes go to out[32..], the payloads to their synchronised offsets;
+ * returns the payload bytes (the sum of CmpL). */
+uint64_t encode_and_place(const int32_t* l, uint64_t nb, int L, uint8_t* out) {
   /* (2) Fixed-length encoding: F_k and CmpL_k per block,
    *     giving the BlockOffsetArray. */
   std::vector<std::vector<uint8_t>> encoded(static_cast<size_t>(nb));
@@ -122,10 +134,7 @@ int compress_with_eb(const float* x, uint64_t n, float eb_abs, float eb_in, int 
   for (uint64_t k = 0; k < nb; ++k)
     if (block_offset[k] > 0)
       std::memcpy(out + p0 + sync_offset[k], encoded[k].data(), size_t(block_offset[k]));
-
-  write_header(out, n, mode, ORACLE_OK, eb_abs, eb_in, payload_bytes, L);
-  *out_bytes = p0 + payload_bytes;
-  return ORACLE_OK;
+  return payload_bytes;
 }
 
 }  // namespace
@@ -390,6 +399,185 @@ int oracle_decompress(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t
       if (idx < n) out[idx] = float(r) * two_eb;
     }
   }
+  return ORACLE_OK;
+}
+
+/* ---- multi-dimensional Lorenzo inside blocks (DESIGN R18) ---- */
+
+namespace {
+
+/* block box (bz, by, bx) of the dims-D predictor: 1x4x8 (2D), 2x4x4 (3D) */
+void md_box(int dims, int* bz, int* by, int* bx) {
+  *bz = (dims == 3) ? 2 : 1;
+  *by = 4;
+  *bx = (dims == 3) ? 4 : 8;
+}
+
+uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+bool md_args_ok(uint64_t nz, uint64_t ny, uint64_t nx, int dims) {
+  return (dims == 2 || dims == 3) && nz > 0 && ny > 0 && nx > 0;
+}
+
+}  // namespace
+
+uint64_t oracle_num_blocks_md(uint64_t nz, uint64_t ny, uint64_t nx, int dims) {
+  int bz, by, bx;
+  md_box(dims, &bz, &by, &bx);
+  return ceil_div(nz, bz) * ceil_div(ny, by) * ceil_div(nx, bx);
+}
+
+uint64_t oracle_max_compressed_bytes_md(uint64_t nz, uint64_t ny, uint64_t nx, int dims) {
+  const uint64_t nb = oracle_num_blocks_md(nz, ny, nx, dims);
+  return HEADER_BYTES + align16(nb) + uint64_t(L / 8) * uint64_t(MAX_F + 1) * nb;
+}
+
+void oracle_block_lorenzo_md(const int32_t r[32], int dims, int32_t l[32]) {
+  /* The Lorenzo predictor (ref [14]) restricted to the block: every
+   * neighbour outside the block counts as 0. */
+  int bz, by, bx;
+  md_box(dims, &bz, &by, &bx);
+  auto at = [&](int z, int y, int x) -> int32_t {
+    if (z < 0 || y < 0 || x < 0) return 0;
+    return r[(z * by + y) * bx + x];
+  };
+  for (int z = 0; z < bz; ++z)
+    for (int y = 0; y < by; ++y)
+      for (int x = 0; x < bx; ++x) {
+        int32_t pred;
+        if (dims == 2)
+          pred = at(z, y, x - 1) + at(z, y - 1, x) - at(z, y - 1, x - 1);
+        else
+          pred = at(z, y, x - 1) + at(z, y - 1, x) + at(z - 1, y, x)
+                 - at(z, y - 1, x - 1) - at(z - 1, y, x - 1) - at(z - 1, y - 1, x)
+                 + at(z - 1, y - 1, x - 1);
+        l[(z * by + y) * bx + x] = at(z, y, x) - pred;
+      }
+}
+
+int oracle_compress_md(const float* x, uint64_t nz, uint64_t ny, uint64_t nx, int dims, float eb,
+                       int mode, uint8_t* out, uint64_t cap, uint64_t* out_bytes) {
+  if (x == nullptr || out == nullptr || out_bytes == nullptr || !md_args_ok(nz, ny, nx, dims))
+    return ORACLE_EINVAL;
+  const uint64_t n = nz * ny * nx;
+  const uint64_t nb = oracle_num_blocks_md(nz, ny, nx, dims);
+  if (cap < oracle_max_compressed_bytes_md(nz, ny, nx, dims)) return ORACLE_ENOSPACE;
+  const int mode_byte = mode | ((dims - 1) << 5);      /* header: predictor dimension (R18) */
+  /* eb_abs exactly as the 1D path (Eq 1, R3) */
+  float eb_abs;
+  if (mode == 0) {
+    if (!eb_usable(eb)) return ORACLE_EINVAL;
+    eb_abs = eb;
+  } else if (mode == 1) {
+    if (!(eb > 0.0f) || !std::isfinite(eb)) return ORACLE_EINVAL;
+    float mn, mx;
+    oracle_value_range(x, size_t(n), &mn, &mx);
+    eb_abs = eb * (mx - mn);
+  } else {
+    return ORACLE_EINVAL;
+  }
+  std::memset(out, 0, size_t(HEADER_BYTES + align16(nb)));
+  if (!eb_usable(eb_abs)) {                             /* R5 */
+    write_header(out, n, mode_byte, ORACLE_ERANGE, eb_abs, eb, 0, L);
+    *out_bytes = HEADER_BYTES + align16(nb);
+    return ORACLE_ERANGE;
+  }
+  /* (1) pre-quantisation of every point, the guard of R18 */
+  std::vector<int32_t> r(static_cast<size_t>(n));
+  if (prequantize_guarded(x, size_t(n), eb_abs, r.data(), dims == 2 ? GUARD2 : GUARD2 / 2) != ORACLE_OK) {
+    write_header(out, n, mode_byte, ORACLE_ERANGE, eb_abs, eb, 0, L);
+    *out_bytes = HEADER_BYTES + align16(nb);
+    return ORACLE_ERANGE;
+  }
+  /* (1') blocks of the field in raster order, zero outside the field, then
+   *      the block-local multi-dimensional Lorenzo prediction */
+  int bz, by, bx;
+  md_box(dims, &bz, &by, &bx);
+  const uint64_t nbz = ceil_div(nz, bz), nby = ceil_div(ny, by), nbx = ceil_div(nx, bx);
+  std::vector<int32_t> l(static_cast<size_t>(nb * L));
+  uint64_t k = 0;
+  for (uint64_t kz = 0; kz < nbz; ++kz)
+    for (uint64_t ky = 0; ky < nby; ++ky)
+      for (uint64_t kx = 0; kx < nbx; ++kx, ++k) {
+        int32_t rb[32];
+        for (int z = 0; z < bz; ++z)
+          for (int y = 0; y < by; ++y)
+            for (int xx = 0; xx < bx; ++xx) {
+              const uint64_t gz = kz * bz + z, gy = ky * by + y, gx = kx * bx + xx;
+              rb[(z * by + y) * bx + xx] =
+                  (gz < nz && gy < ny && gx < nx) ? r[size_t((gz * ny + gy) * nx + gx)] : 0;
+            }
+        oracle_block_lorenzo_md(rb, dims, &l[size_t(k * L)]);
+      }
+  /* (2)-(4) exactly as the 1D path */
+  const uint64_t payload_bytes = encode_and_place(l.data(), nb, L, out);
+  write_header(out, n, mode_byte, ORACLE_OK, eb_abs, eb, payload_bytes, L);
+  *out_bytes = HEADER_BYTES + align16(nb) + payload_bytes;
+  return ORACLE_OK;
+}
+
+int oracle_decompress_md(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t nz,
+                         uint64_t ny, uint64_t nx, int dims) {
+  if (in == nullptr || out == nullptr || !md_args_ok(nz, ny, nx, dims)) return ORACLE_EINVAL;
+  if (in_bytes < uint64_t(HEADER_BYTES)) return ORACLE_ECORRUPT;
+  if (!(in[0] == 'C' && in[1] == 'S' && in[2] == 'Z' && in[3] == 'P') || in[4] != 1 || in[7] != 5 ||
+      ((in[5] >> 5) & 3) != dims - 1 || (in[5] & 0x10))
+    return ORACLE_ECORRUPT;
+  if (in[6] != ORACLE_OK) return in[6] == ORACLE_ERANGE ? ORACLE_ERANGE : ORACLE_ECORRUPT;
+  const uint64_t n = nz * ny * nx;
+  if (get_u64(in + 8) != n) return ORACLE_EINVAL;
+  const float eb_abs = get_f32(in + 16);
+  const uint64_t payload_bytes = get_u64(in + 24);
+  const uint64_t nb = oracle_num_blocks_md(nz, ny, nx, dims);
+  const uint64_t p0 = HEADER_BYTES + align16(nb);
+  if (in_bytes < p0 || !eb_usable(eb_abs)) return ORACLE_ECORRUPT;
+  /* F -> CmpL (Eq 2) -> offsets (Eq 3), as the 1D path */
+  const uint8_t* fixed_length = in + HEADER_BYTES;
+  std::vector<uint64_t> block_offset(static_cast<size_t>(nb)), sync_offset(static_cast<size_t>(nb));
+  for (uint64_t k = 0; k < nb; ++k) {
+    if (fixed_length[k] > MAX_F) return ORACLE_ECORRUPT;
+    block_offset[k] = oracle_block_bytes(fixed_length[k], L);
+  }
+  oracle_exclusive_scan(block_offset.data(), size_t(nb), sync_offset.data());
+  if (sync_offset[nb - 1] + block_offset[nb - 1] != payload_bytes || in_bytes < p0 + payload_bytes)
+    return ORACLE_ECORRUPT;
+  int bz, by, bx;
+  md_box(dims, &bz, &by, &bx);
+  const uint64_t nbz = ceil_div(nz, bz), nby = ceil_div(ny, by), nbx = ceil_div(nx, bx);
+  const float two_eb = eb_abs + eb_abs;
+  uint64_t k = 0;
+  for (uint64_t kz = 0; kz < nbz; ++kz)
+    for (uint64_t ky = 0; ky < nby; ++ky)
+      for (uint64_t kx = 0; kx < nbx; ++kx, ++k) {
+        int32_t l[32], r[32];
+        oracle_decode_block_L(in + p0 + sync_offset[k], fixed_length[k], L, l);
+        /* inverse prediction, in the block's raster order: r = l + pred(r),
+         * the predictor's neighbours all precede the point */
+        for (int z = 0; z < bz; ++z)
+          for (int y = 0; y < by; ++y)
+            for (int xx = 0; xx < bx; ++xx) {
+              auto at = [&](int zz, int yy, int x2) -> int32_t {
+                if (zz < 0 || yy < 0 || x2 < 0) return 0;
+                return r[(zz * by + yy) * bx + x2];
+              };
+              int32_t pred;
+              if (dims == 2)
+                pred = at(z, y, xx - 1) + at(z, y - 1, xx) - at(z, y - 1, xx - 1);
+              else
+                pred = at(z, y, xx - 1) + at(z, y - 1, xx) + at(z - 1, y, xx)
+                       - at(z, y - 1, xx - 1) - at(z - 1, y, xx - 1) - at(z - 1, y - 1, xx)
+                       + at(z - 1, y - 1, xx - 1);
+              r[(z * by + y) * bx + xx] = l[(z * by + y) * bx + xx] + pred;
+            }
+        /* d' = r * 2eb at the points inside the field */
+        for (int z = 0; z < bz; ++z)
+          for (int y = 0; y < by; ++y)
+            for (int xx = 0; xx < bx; ++xx) {
+              const uint64_t gz = kz * bz + z, gy = ky * by + y, gx = kx * bx + xx;
+              if (gz < nz && gy < ny && gx < nx)
+                out[size_t((gz * ny + gy) * nx + gx)] = float(r[(z * by + y) * bx + xx]) * two_eb;
+            }
+      }
   return ORACLE_OK;
 }
 

@@ -116,6 +116,30 @@ int oracle_compress_minmax_L(const float* x, uint64_t n, float lambda,
 int oracle_compress_ex(const float* x, uint64_t n, float eb, int mode, int L, int order,
                        uint8_t* out, uint64_t cap, uint64_t* out_bytes);
 
+/* ---- multi-dimensional Lorenzo inside blocks -----
+ * "Lorenzo predictions with higher dimensions" (the Lorenzo
+ * predictor of ref [14]), DESIGN R18.  The field has shape (nz, ny, nx), x
+ * fastest, n = nz*ny*nx.  An L = 32 block is a 1 x 4 x 8 (dims = 2) or
+ * 2 x 4 x 4 (dims = 3) box of the field; blocks tile the field in raster
+ * order of the block grid (ceil(nz/bz), ceil(ny/4), ceil(nx/bx)), x
+ * fastest; element j of a block is (z*4 + y)*bx + x.  Elements outside the
+ * field are quantisation integer 0 (R8), and the predictor treats
+ * neighbours outside the BLOCK as 0 (block-local, like P:525-529):
+ *   dims 2: l = r - r(y,x-1) - r(y-1,x) + r(y-1,x-1)
+ *   dims 3: l = r - r(x-1) - r(y-1) - r(z-1) + r(y-1,x-1) + r(z-1,x-1)
+ *               + r(z-1,y-1) - r(z-1,y-1,x-1)            (same z/y/x otherwise)
+ * Guard |r0| < 2^21 (dims 2) or 2^20 (dims 3) so |l| < 2^23 and F <= 24.
+ * Stream: the L = 32 format with nb = the number of grid blocks, header
+ * mode byte bits 5-6 = dims - 1; the shape is the caller's (like n).
+ * dims = 1 is oracle_compress (the 1D predictor, blocks of 32 in order). */
+uint64_t oracle_num_blocks_md(uint64_t nz, uint64_t ny, uint64_t nx, int dims);
+uint64_t oracle_max_compressed_bytes_md(uint64_t nz, uint64_t ny, uint64_t nx, int dims);
+void oracle_block_lorenzo_md(const int32_t r[32], int dims, int32_t l[32]);
+int oracle_compress_md(const float* x, uint64_t nz, uint64_t ny, uint64_t nx, int dims, float eb,
+                       int mode, uint8_t* out, uint64_t cap, uint64_t* out_bytes);
+int oracle_decompress_md(const uint8_t* in, uint64_t in_bytes, float* out, uint64_t nz,
+                         uint64_t ny, uint64_t nx, int dims);
+
 /* ---- reconstruction quality -------------------
  * The statistics of the paper's artifact output (QCAT compareData,
  * P:1918-1933) and PSNR (sec 2.1), in fp64, two plain passes

@@ -88,7 +88,7 @@ struct CompressSmem {
 };
 
 __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
-  return *reinterpret_cast<const volatile uint32_t*>(p);
+  return *reinterpret_cast<const volatile uint32_t*>(p);  // sync: flag poll (ring tail / released), ordered by the writer's fence
 }
 
 // R2 op sequence with explicit RN intrinsics (never contracted further):
@@ -279,19 +279,19 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           stress_delay(i);
           const uint32_t t = atomicAdd(&a.ws->ticket, 1u);
           if (t >= a.num_tiles) {
-            sm.in_tile[s] = kSentinel;
+            sm.in_tile[s] = kSentinel;  // sync: mbarrier full[s] (arrive release / try_wait acquire)
             mbar_arrive(&sm.full[s]);
             // every writer must see a sentinel: one in each of the next kWriters ticket slots
             for (uint32_t k = 0; k < uint32_t(kWriters); ++k) {
-              sm.tix[(i + k) % kTix] = kSentinel;
+              sm.tix[(i + k) % kTix] = kSentinel;  // sync: mbarrier tixbar
               mbar_arrive(&sm.tixbar[(i + k) % kTix]);
             }
             break;
           }
-          sm.tix[i % kTix] = t;                          // writers start the look-back now
+          sm.tix[i % kTix] = t;                          // writers start the look-back now  // sync: mbarrier tixbar
           mbar_arrive(&sm.tixbar[i % kTix]);
           trace_put(a.trace, t, 0, global_ns());
-          sm.in_tile[s] = t;
+          sm.in_tile[s] = t;  // sync: mbarrier full[s]
           const uint64_t e0 = uint64_t(t) * kTileElems;
           const uint64_t ne = min(uint64_t(kTileElems), a.n - e0);
           const uint32_t bytes = uint32_t(ne * 4);
@@ -311,7 +311,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         // exclusive prefix (the look-back needs only the predecessors' words)
         // while the tile is still loading and being encoded
         mbar_wait(&sm.tixbar[j % kTix], (j / kTix) & 1u);
-        const uint32_t t = sm.tix[j % kTix];
+        const uint32_t t = sm.tix[j % kTix];  // sync: mbarrier tixbar
         if (t == kSentinel) break;
         uint32_t nw = 0, ns = 0;
 #if CUSZP_C_LB_DELAY > 0
@@ -332,7 +332,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           // counts, F = words - 1 (0 for a zero block) bytewise (counts <= 32, no
           // carries); the stores also cover the F area's zero padding up to
           // align16(nb) (sub-blocks past n encode as zero blocks, F = 0)
-          const uint32_t wb = md.wb[lane];
+          const uint32_t wb = md.wb[lane];  // sync: mbarrier staged[m] after the compute warps' acq_rel count
           uint32_t f = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
           const uint64_t blk = (uint64_t(t) * kTileBlocks + 4u * lane) / M;
           if (blk < align16(a.nb)) {
@@ -341,8 +341,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             else a.out[kHdr + blk] = uint8_t(f);
           }
         }
-        const uint32_t cnt = lane < kCW ? md.cnt[lane] : 0u;
-        const uint32_t hd = lane < kCW ? md.head[lane] : 0u;
+        const uint32_t cnt = lane < kCW ? md.cnt[lane] : 0u;  // sync: mbarrier staged[m]
+        const uint32_t hd = lane < kCW ? md.head[lane] : 0u;  // sync: mbarrier staged[m]
         uint32_t incl = cnt;
 #pragma unroll
         for (int o = 1; o < kCW; o <<= 1) {
@@ -370,21 +370,21 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           uint32_t* dst = dst_t + off;
           const uint32_t* src = sm.ring[w] + h + lane;
 #pragma unroll 4
-          for (int k = lane; k < int(first); k += 32, src += 32, dst += 32) *dst = *src;
+          for (int k = lane; k < int(first); k += 32, src += 32, dst += 32) *dst = *src;  // sync: ring written before staged[m]; reused only after the tail release
           src = sm.ring[w] + lane;
           dst = dst_t + off + first;
 #pragma unroll 2
-          for (int k = lane; k < int(c - first); k += 32, src += 32, dst += 32) *dst = *src;
+          for (int k = lane; k < int(c - first); k += 32, src += 32, dst += 32) *dst = *src;  // sync: ring written before staged[m]; reused only after the tail release
         }
         // release ring space in CTA tile order
         if (lane == 0) stress_delay(j ^ 0x55u);
         __syncwarp();
         while (ld_volatile_u32(&sm.released) != j) __nanosleep(64);
-        if (lane < kCW) sm.tail[lane] += cnt;
+        if (lane < kCW) sm.tail[lane] += cnt;  // sync: released in tile order after the copy (fence + volatile flag)
         __syncwarp();
         if (lane == 0) {
           __threadfence_block();
-          *reinterpret_cast<volatile uint32_t*>(&sm.released) = j + 1;
+          *reinterpret_cast<volatile uint32_t*>(&sm.released) = j + 1;  // sync: fence + volatile flag, polled by the compute warps
         }
         __syncwarp();
       }
@@ -402,7 +402,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
         mbar_wait(&sm.full[s], (i / kStages) & 1u);         // suspending wait: no issue slots taken
-        const uint32_t t = sm.in_tile[s];
+        const uint32_t t = sm.in_tile[s];  // sync: mbarrier full[s]
 #ifdef CUSZP_TRACE
         // (diagnostics build only: a lane-0 branch here makes ptxas treat the
         // whole encode as possibly divergent -- a divergence check before every
@@ -534,41 +534,41 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
               const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
               const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
-              if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;
+              if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             } else if (span <= 16) {
               const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
               const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
               const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
-              if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;
+              if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
               const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
               const uint32_t sub23 = (M == 2) ? h : 2u + h;
-              if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;
+              if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             } else {
 #pragma unroll
               for (int q = 0; q < 4; ++q) {
                 const uint32_t tq = xpose(v[q]);
                 const uint32_t pre = (q & ~(M - 1)) == 0 ? 0u : __byte_perm(pb, 0, 0x4440u + (q & ~(M - 1)));
-                if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;
+                if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
               }
             }
           } else if (span <= 8) {
             const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
             const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
-            if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;
+            if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
           } else if (span <= 16) {
             const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
             const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
             const bool hi = lane >= 16;
             const uint32_t k = lane & 15;
-            if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;
-            if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;
+            if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+            if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
           } else {
             uint32_t o = base;
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
               const uint32_t tq = xpose(v[q]);
-              if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;
+              if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
               o += wq[q];
             }
           }
@@ -580,10 +580,10 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
           TileMeta& md = sm.meta[m];
           // the group word counts go to the writer, which stores the tile's F bytes
-          if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);
-          else *reinterpret_cast<uint2*>(&md.wb[w * 2]) = make_uint2(wbs[0], wbs[1]);
-          md.cnt[w] = uint16_t(cursor);
-          md.head[w] = uint16_t(head & (kRing - 1));
+          if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
+          else *reinterpret_cast<uint2*>(&md.wb[w * 2]) = make_uint2(wbs[0], wbs[1]);  // sync: acq_rel count, then mbarrier staged[m]
+          md.cnt[w] = uint16_t(cursor);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
+          md.head[w] = uint16_t(head & (kRing - 1));  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           uint32_t done;                                   // release: cnt/head before the count; acquire: the others'
           asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
                        : "=r"(done) : "r"(smem_u32(&sm.meta_done[m])) : "memory");
@@ -592,7 +592,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             uint32_t agg = 0;
 #pragma unroll
             for (int k = 0; k < kCW; ++k)
-              agg += *reinterpret_cast<volatile uint16_t*>(&md.cnt[k]);
+              agg += *reinterpret_cast<volatile uint16_t*>(&md.cnt[k]);  // sync: atom.acq_rel on meta_done[m] (the last warp acquires every warp's count)
             publish_aggregate(a.status, t, agg, epoch);
             trace_put(a.trace, t, 2, global_ns());
             md.tile = t;

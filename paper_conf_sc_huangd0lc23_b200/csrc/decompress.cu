@@ -238,7 +238,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           const int s = int(k % kDStages);
           if (k >= uint32_t(kDStages)) named_sync(kBarEmpty0 + s, kBarCount);
           if (lane == 0) {
-            sm.tile[s] = kSentinel;
+            sm.tile[s] = kSentinel;  // sync: mbarrier full[s]
             mbar_arrive(&sm.full[s]);
           }
           break;
@@ -246,7 +246,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
         for (uint32_t j = 0; j < cd.ntiles; ++j) {
           const int s = int(k % kDStages);
           if (k >= uint32_t(kDStages)) named_sync(kBarEmpty0 + s, kBarCount);
-          sm.ginfo[s][lane] = make_uint2(cd.gwords[j][lane], cd.gmeta[j][lane]);
+          sm.ginfo[s][lane] = make_uint2(cd.gwords[j][lane], cd.gmeta[j][lane]);  // sync: mbarrier full[s]; reused after the EMPTY named barrier
           const uint64_t tw = cd.tile_words[j];
           uint32_t tma_bytes = 0, delta = 0;
           uint64_t a0 = 0;
@@ -260,12 +260,12 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             // words past the last full 16 bytes inside in_bytes (<= 3)
             const uint64_t tail_words = end > a1 ? (end - a1) / 4 : 0;
             if (uint64_t(lane) < tail_words)
-              sm.data[s][(a1 - a0) / 4 + lane] = *reinterpret_cast<const uint32_t*>(a.in + a1 + 4 * lane);
+              sm.data[s][(a1 - a0) / 4 + lane] = *reinterpret_cast<const uint32_t*>(a.in + a1 + 4 * lane);  // sync: mbarrier full[s]
           }
           __syncwarp();
           if (lane == 0) {
-            sm.tile[s] = cd.chunk * kChunkTiles + j;
-            sm.delta[s] = delta;
+            sm.tile[s] = cd.chunk * kChunkTiles + j;  // sync: mbarrier full[s]
+            sm.delta[s] = delta;  // sync: mbarrier full[s]
             mbar_arrive_expect_tx(&sm.full[s], tma_bytes);   // one phase per use, even with 0 bytes
             if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
           }
@@ -295,10 +295,10 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kDStages);
         mbar_wait(&sm.full[s], (i / kDStages) & 1u);          // tile's payload landed (suspending wait)
-        const uint32_t t = sm.tile[s];
+        const uint32_t t = sm.tile[s];  // sync: mbarrier full[s]
         if (t == kSentinel) break;
         const bool last = (t == a.num_tiles - 1);
-        const uint32_t* data = sm.data[s] + sm.delta[s];
+        const uint32_t* data = sm.data[s] + sm.delta[s];  // sync: mbarrier full[s]
         float* outp = a.out + uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32 + q * 32u + lane4;
 #pragma unroll kDUnroll
 #ifdef CUSZP_DIAG_NOWORK
@@ -306,7 +306,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 #else
         for (int g = 0; g < kBPW / 4; ++g) {
 #endif
-          const uint2 gi = sm.ginfo[s][w * 4 + g];
+          const uint2 gi = sm.ginfo[s][w * 4 + g];  // sync: mbarrier full[s]
           const uint32_t wbytes = gi.x;
           const uint32_t* gdata = data + (gi.y & 0xffffu);
           const uint32_t mode = gi.y >> 16;

@@ -61,3 +61,32 @@ def decode_to_floats(buf: bytes):
     two_eb = np.float32(h["eb_abs"]) + np.float32(h["eb_abs"])
     q = np.array(r[: h["n"]], dtype=np.float32)
     return h, (q * two_eb).astype(np.float32)
+
+
+def decode_l_blocks(buf: bytes, nb: int) -> tuple[dict, list[int], list[list[int]]]:
+    """The Lorenzo integers l of each of nb L-blocks (no inverse prediction):
+    for streams whose block count is not ceil(n / L), e.g. the
+    multi-dimensional predictor's block grid (DESIGN R18)."""
+    h = parse_header(buf)
+    Lb = 1 << h["log2l"]
+    F = list(buf[32:32 + nb])
+    pos = 32 + ((nb + 15) // 16) * 16
+    out = []
+    for k in range(nb):
+        f = F[k]
+        if f == 0:
+            out.append([0] * Lb)
+            continue
+        nbytes = (f + 1) * Lb // 8
+        blk = buf[pos:pos + nbytes]
+        pos += nbytes
+        ls = []
+        for j in range(Lb):
+            neg = (blk[j // 8] >> (j % 8)) & 1
+            mag = 0
+            for p in range(f):
+                mag |= ((blk[(p + 1) * (Lb // 8) + j // 8] >> (j % 8)) & 1) << p
+            ls.append(-mag if neg else mag)
+        out.append(ls)
+    h["consumed"] = pos
+    return h, F, out
