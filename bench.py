@@ -599,6 +599,39 @@ def variants(r: Runner, peak: float, steps: int) -> dict:
             "decompress_frac_of_peak": round((4 * n0 + SL) / tdm / 1e9 / peak, 4)}
         if outL is not r.out:
             del outL
+    # multi-dimensional Lorenzo on the same field as
+    # a (100, 500, 500) volume: 2D (1x4x8 blocks) and 3D (2x4x4 blocks)
+    shape = (100, 500, 500)
+    for dims in (2, 3):
+        capm = int(lib.cuszp_max_compressed_bytes_md(*shape, dims))
+        wsm = cz.WorkspaceMD(shape, dims, r.dev)
+        outm = r.out if capm <= r.cap else torch.empty(capm, dtype=torch.uint8, device=r.dev)
+        tc, td = [], []
+        for _ in range(steps + 1):
+            r.flush_l2()
+            ev[0].record(r.stream)
+            cz.check(lib.cuszp_compress_md(x0.data_ptr(), *shape, dims, eb_abs, cz.ABS, outm.data_ptr(), capm,
+                                           r.out_bytes.data_ptr(), wsm.ptr(), wsm.nbytes, sp), "compress_md")
+            ev[1].record(r.stream)
+            torch.cuda.synchronize(r.dev)
+            tc.append(ev[0].elapsed_time(ev[1]))
+            r.flush_l2()
+            ev[0].record(r.stream)
+            cz.check(lib.cuszp_decompress_md(outm.data_ptr(), capm, r.y.data_ptr(), *shape, dims, wsm.ptr(),
+                                             wsm.nbytes, sp), "decompress_md")
+            ev[1].record(r.stream)
+            torch.cuda.synchronize(r.dev)
+            td.append(ev[0].elapsed_time(ev[1]))
+        assert cz.last_status(wsm) == cz.OK
+        SL = int(r.out_bytes.item())
+        tcm, tdm = float(np.median(tc[1:])) / 1e3, float(np.median(td[1:])) / 1e3
+        out[f"32_lorenzo{dims}d"] = {
+            "cr": round(4 * n0 / SL, 3),
+            "compress_kernel_gbs": round(4 * n0 / tcm / 1e9, 1),
+            "decompress_kernel_gbs": round(4 * n0 / tdm / 1e9, 1),
+            "compress_frac_of_peak": round((4 * n0 + SL) / tcm / 1e9 / peak, 4),
+            "decompress_frac_of_peak": round((4 * n0 + SL) / tdm / 1e9 / peak, 4)}
+        del wsm
     del x0
     torch.cuda.empty_cache()
     return out

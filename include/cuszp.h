@@ -200,6 +200,31 @@ int cuszp_decompress_host_async(const void* h_in, size_t in_capacity, float* h_o
                                 void* d_in_scratch, float* d_out_scratch,
                                 void* d_ws, size_t ws_bytes, void* stream);
 
+/* ---- multi-dimensional Lorenzo ----
+ * "Lorenzo predictions with higher dimensions" inside blocks (DESIGN R18).
+ * The field is an (nz, ny, nx) array, x fastest, n = nz*ny*nx (nz = 1 for a
+ * 2D field).  dims = 2: an L = 32 block is a 1 x 4 x 8 box of the field,
+ * dims = 3: a 2 x 4 x 4 box; blocks tile the field in raster order of the
+ * block grid (x fastest), points outside the field are quantisation
+ * integer 0 (R8), and the block-local predictor takes neighbours outside
+ * the block as 0:  dims 2: l = r - r(x-1) - r(y-1) + r(y-1,x-1);  dims 3:
+ * the 7-term Lorenzo predictor.  Guard |round(d/2eb)| < 2^21 (dims 2) or
+ * 2^20 (dims 3), else ERANGE.  Stream: the L = 32 format with nb =
+ * cuszp_num_blocks_md() blocks; header mode byte bits 5-6 = dims - 1.  The
+ * shape is not stored: decompression takes it (like n).  Buffers: output
+ * cuszp_max_compressed_bytes_md, workspace cuszp_workspace_bytes_md (zeroed
+ * once, like every workspace).  Sync errors: EINVAL (dims not 2 or 3, a zero
+ * extent, > 2^32 blocks, NULL / misaligned pointers, eb as for
+ * cuszp_compress), ENOSPACE, ECUDA; data errors asynchronous as usual. */
+size_t cuszp_num_blocks_md(size_t nz, size_t ny, size_t nx, int dims);
+size_t cuszp_max_compressed_bytes_md(size_t nz, size_t ny, size_t nx, int dims);
+size_t cuszp_workspace_bytes_md(size_t nz, size_t ny, size_t nx, int dims);
+int cuszp_compress_md(const float* d_in, size_t nz, size_t ny, size_t nx, int dims, float eb, int mode,
+                      void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
+                      void* d_ws, size_t ws_bytes, void* stream);
+int cuszp_decompress_md(const void* d_in, size_t in_bytes, float* d_out, size_t nz, size_t ny, size_t nx,
+                        int dims, void* d_ws, size_t ws_bytes, void* stream);
+
 /* ---- reconstruction quality on the device ----
  * The statistics the paper's artifact reads off QCAT compareData
  * (P:1918-1933), PSNR as in sec 2.1, all in fp64.  x = original,

@@ -29,7 +29,7 @@ __all__ = [
     "ABS", "REL", "Workspace", "compress", "compress_minmax", "decompress", "value_range",
     "max_compressed_bytes", "workspace_bytes", "last_status", "read_header", "compress_host",
     "decompress_host", "CuszpError", "exact_bytes_from_F", "quality", "QUALITY_KEYS",
-    "compress_host_async", "decompress_host_async",
+    "compress_host_async", "decompress_host_async", "compress_md", "decompress_md", "WorkspaceMD",
 ]
 
 
@@ -192,6 +192,77 @@ def decompress(stream_buf: torch.Tensor, n: int, out: torch.Tensor | None = None
         raise ValueError(f"in_bytes={nbytes} exceeds the stream buffer ({stream_buf.numel()} bytes)")
     check(lib().cuszp_decompress_ex(stream_buf.data_ptr(), nbytes, out.data_ptr(), int(n), int(block_len),
                                     int(order), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_decompress")
+    return out
+
+
+def _shape3(shape) -> tuple[int, int, int]:
+    shape = tuple(int(v) for v in shape)
+    if not 1 <= len(shape) <= 3:
+        raise ValueError("shape must have 1 to 3 dimensions")
+    return (1,) * (3 - len(shape)) + shape
+
+
+class WorkspaceMD(Workspace):
+    """Zeroed workspace for the multi-dimensional calls on a given shape."""
+
+    def __init__(self, shape, dims: int, device=None):
+        device = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        nz, ny, nx = _shape3(shape)
+        self.n = nz * ny * nx
+        self.nbytes = int(lib().cuszp_workspace_bytes_md(nz, ny, nx, int(dims)))
+        if self.nbytes == 0:
+            raise ValueError("unsupported shape / dims")
+        self.buf = torch.zeros(self.nbytes, dtype=torch.uint8, device=device)
+
+
+def compress_md(x: torch.Tensor, eb: float, mode="rel", dims: int | None = None, shape=None,
+                out: torch.Tensor | None = None, out_bytes: torch.Tensor | None = None, ws: Workspace | None = None,
+                stream=None):
+    """Compress a 2D/3D float32 CUDA field with the multi-dimensional Lorenzo
+    predictor (dims 2: 1x4x8 blocks, 3: 2x4x4 blocks; DESIGN R18).  shape
+    defaults to x.shape, dims to len(shape).  Returns (stream buffer, device
+    int64[1] stream length)."""
+    _require_cuda(x, "x", torch.float32)
+    shape = tuple(x.shape) if shape is None else tuple(shape)
+    nz, ny, nx = _shape3(shape)
+    if nz * ny * nx != x.numel():
+        raise ValueError("shape does not match x")
+    dims = len(shape) if dims is None else int(dims)
+    cap = int(lib().cuszp_max_compressed_bytes_md(nz, ny, nx, dims))
+    if cap == 0:
+        raise ValueError("unsupported shape / dims")
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, device=x.device)
+    _require_cuda(out, "out", torch.uint8)
+    if out_bytes is None:
+        out_bytes = torch.zeros(1, dtype=torch.int64, device=x.device)
+    _check_out_bytes(out_bytes)
+    if ws is None:
+        ws = WorkspaceMD(shape, dims, x.device)
+    check(lib().cuszp_compress_md(x.data_ptr(), nz, ny, nx, dims, float(eb), _mode(mode), out.data_ptr(), out.numel(),
+                                  out_bytes.data_ptr(), ws.ptr(), ws.nbytes, _stream_ptr(stream)), "cuszp_compress_md")
+    return out, out_bytes
+
+
+def decompress_md(stream_buf: torch.Tensor, shape, dims: int | None = None, out: torch.Tensor | None = None,
+                  in_bytes: int | None = None, ws: Workspace | None = None, stream=None) -> torch.Tensor:
+    """Decompress a multi-dimensional-Lorenzo stream into a field of the given shape."""
+    _require_cuda(stream_buf, "stream_buf", torch.uint8)
+    shape = tuple(int(v) for v in shape)
+    nz, ny, nx = _shape3(shape)
+    dims = len(shape) if dims is None else int(dims)
+    if out is None:
+        out = torch.empty(shape, dtype=torch.float32, device=stream_buf.device)
+    _require_cuda(out, "out", torch.float32)
+    if out.numel() < nz * ny * nx:
+        raise ValueError("out is smaller than the field")
+    nbytes = stream_buf.numel() if in_bytes is None else int(in_bytes)
+    if nbytes > stream_buf.numel() or nbytes < 0:
+        raise ValueError("in_bytes exceeds the stream buffer")
+    if ws is None:
+        ws = WorkspaceMD(shape, dims, stream_buf.device)
+    check(lib().cuszp_decompress_md(stream_buf.data_ptr(), nbytes, out.data_ptr(), nz, ny, nx, dims, ws.ptr(),
+                                    ws.nbytes, _stream_ptr(stream)), "cuszp_decompress_md")
     return out
 
 

@@ -26,6 +26,8 @@ SYMBOLS = (
     "cuszp_compress_host_async", "cuszp_decompress_host_async",
     "cuszp_compress_L", "cuszp_compress_minmax_L", "cuszp_decompress_L", "cuszp_max_compressed_bytes_L",
     "cuszp_compress_ex", "cuszp_decompress_ex",
+    "cuszp_num_blocks_md", "cuszp_max_compressed_bytes_md", "cuszp_workspace_bytes_md", "cuszp_compress_md",
+    "cuszp_decompress_md",
 )
 
 _lock = threading.Lock()
@@ -84,6 +86,13 @@ def _declare(h):
     h.cuszp_compress_minmax_L.restype = i32
     h.cuszp_decompress_L.argtypes = [vp, sz, vp, sz, i32, vp, sz, vp]
     h.cuszp_decompress_L.restype = i32
+    for f in ("cuszp_num_blocks_md", "cuszp_max_compressed_bytes_md", "cuszp_workspace_bytes_md"):
+        getattr(h, f).argtypes = [sz, sz, sz, i32]
+        getattr(h, f).restype = sz
+    h.cuszp_compress_md.argtypes = [vp, sz, sz, sz, i32, f32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_compress_md.restype = i32
+    h.cuszp_decompress_md.argtypes = [vp, sz, vp, sz, sz, sz, i32, vp, sz, vp]
+    h.cuszp_decompress_md.restype = i32
     h.cuszp_version.argtypes = []
     h.cuszp_version.restype = i32
 

@@ -218,11 +218,36 @@ __device__ __forceinline__ uint32_t lorenzo2_pack(uint32_t rb, int lane) {
   return (a << 1) | (uint32_t(l) >> 31);
 }
 
+// lane j holds the biased r_j of one block in block order (element j =
+// (z*4 + y)*bx + x) -> v_j for the block-local multi-dimensional Lorenzo
+// (R18), as successive differences along x, y (and z), each taking 0 at the
+// block's edge: 2D (4x8) l = r - r(x-1) - r(y-1) + r(y-1,x-1), 3D (2x4x4) the
+// 7-term predictor.
+template <int D>
+__device__ __forceinline__ uint32_t lorenzo_md_pack(uint32_t rb, int lane) {
+  constexpr int kBX = (D == 3) ? 4 : 8;
+  uint32_t px = __shfl_up_sync(kFull, rb, 1);
+  px = (lane % kBX) ? px : kRoundMagicBits;
+  int l = int(rb - px);                                      // along x; the biases cancel
+  const int uy = __shfl_up_sync(kFull, l, kBX);
+  if ((lane / kBX) % 4) l -= uy;                             // along y
+  if constexpr (D == 3) {
+    const int uz = __shfl_up_sync(kFull, l, 16);
+    if (lane >= 16) l -= uz;                                 // along z
+  }
+  const uint32_t a = uint32_t(l < 0 ? -l : l);
+  return (a << 1) | (uint32_t(l) >> 31);
+}
+
 // O = Lorenzo order: 1 (the paper's 1D 1-layer predictor) or 2 (2-layer,
 // SURVEY 8(f) rank 4; L = 32 only).
-template <int M, int O>
+// D = Lorenzo dimensions (DESIGN R18): 1 = the paper's 1D
+// predictor over consecutive elements; 2 / 3 = blocks of 1x4x8 / 2x4x4 points
+// of an (nz, ny, nx) field, gathered into tile order by the producer warp.
+template <int M, int O, int D = 1>
 __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(CompressArgs a) {
   static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
+  static_assert(D == 1 || (M == 1 && O == 1), "multi-dimensional Lorenzo with L = 32, order 1");
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
   extern __shared__ __align__(128) unsigned char smem_raw[];
   CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
@@ -257,7 +282,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   uint32_t* payload = reinterpret_cast<uint32_t*>(a.out + p0);
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], 1); mbar_init(&sm.empty[s], kCW); }
+    // D > 1: the 32 producer lanes' cp.async groups complete the stage
+    for (int s = 0; s < kStages; ++s) { mbar_init(&sm.full[s], D == 1 ? 1 : 32); mbar_init(&sm.empty[s], kCW); }
     for (int m = 0; m < kMeta; ++m) { mbar_init(&sm.staged[m], 1); sm.meta_done[m] = 0; }
     for (int k = 0; k < kTix; ++k) mbar_init(&sm.tixbar[k], 1);
     for (int w = 0; w < kCW; ++w) sm.tail[w] = 0;
@@ -267,7 +293,86 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   __syncthreads();
 
   if (eb_ok) {
-    if (warp == 0) {
+    if (D > 1 && warp == 0) {
+      // -------------------------------------------- producer, multi-dim blocks
+      // Tile t = blocks 128t .. 128t+127 of the block grid (raster order, x
+      // fastest).  Every lane gathers rows of 4 floats of those blocks into
+      // the stage in BLOCK order (element j of block i at 32 i + j) with
+      // cp.async, zero-filling points outside the field (R8); each lane's
+      // copies then complete one of the stage's 32 arrivals.
+      constexpr int kBX = (D == 3) ? 4 : 8;
+      const bool al16 = (a.nx % 4 == 0) && ((reinterpret_cast<uintptr_t>(a.in) & 15u) == 0);
+      for (uint32_t i = 0;; ++i) {
+        const int s = int(i % kStages);
+        mbar_wait(&sm.empty[s], ((i / kStages) & 1u) ^ 1u);
+        uint32_t t = 0;
+        if (lane == 0) {
+          stress_delay(i);
+          t = atomicAdd(&a.ws->ticket, 1u);
+        }
+        t = __shfl_sync(kFull, t, 0);
+        if (t >= a.num_tiles) {
+          if (lane == 0) {
+            sm.in_tile[s] = kSentinel;  // sync: mbarrier full[s]
+            for (uint32_t k = 0; k < uint32_t(kWriters); ++k) {
+              sm.tix[(i + k) % kTix] = kSentinel;  // sync: mbarrier tixbar
+              mbar_arrive(&sm.tixbar[(i + k) % kTix]);
+            }
+          }
+          __syncwarp();
+          mbar_arrive(&sm.full[s]);
+          break;
+        }
+        if (lane == 0) {
+          sm.tix[i % kTix] = t;  // sync: mbarrier tixbar
+          mbar_arrive(&sm.tixbar[i % kTix]);
+          sm.in_tile[s] = t;  // sync: mbarrier full[s]
+        }
+        const uint32_t dst0 = smem_u32(sm.in[s]);
+        // lane l gathers blocks l, l+32, l+64, l+96 of the tile (neighbouring
+        // lanes read neighbouring row segments); block coordinates from one
+        // 32-bit division per block (nb < 2^32, checked on the host)
+#pragma unroll 1
+        for (uint32_t ib = lane; ib < uint32_t(kTileBlocks); ib += 32) {
+          const uint32_t b = t * uint32_t(kTileBlocks) + ib;
+          const uint32_t nbx = uint32_t(a.nbx), nby = uint32_t(a.nby);
+          const uint32_t kyz = b / nbx, kx = b - kyz * nbx;
+          const uint32_t kz = kyz / nby, ky = kyz - kz * nby;
+          const bool blk_in = uint64_t(b) < a.nb;
+#pragma unroll
+          for (uint32_t r = 0; r < 8; ++r) {                          // the block's 8 row segments of 4 points
+            uint64_t gz, gy, gx;
+            uint32_t d;                                                // element index in the block
+            if constexpr (D == 2) {
+              gz = kz; gy = uint64_t(ky) * 4 + (r >> 1); gx = uint64_t(kx) * 8 + 4 * (r & 1u);
+              d = (r >> 1) * 8 + 4 * (r & 1u);
+            } else {
+              gz = uint64_t(kz) * 2 + (r >> 2); gy = uint64_t(ky) * 4 + (r & 3u); gx = uint64_t(kx) * 4;
+              d = r * 4;
+            }
+            const bool row_in = blk_in && gz < a.nz && gy < a.ny;
+            const float* src = a.in + (row_in ? (gz * a.ny + gy) * a.nx + gx : 0);
+            const uint32_t dst = dst0 + 4u * (ib * 32u + d);
+            if (al16) {
+              const uint32_t bytes = (row_in && gx < a.nx) ? 16u : 0u;   // nx % 4 == 0: a row of 4 is all in or all out
+              asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(bytes ? src : a.in),
+                           "r"(bytes)
+                           : "memory");
+            } else {
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const uint32_t bytes = (row_in && gx + e < a.nx) ? 4u : 0u;
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(dst + 4 * e),
+                             "l"(bytes ? src + e : a.in), "r"(bytes)
+                             : "memory");
+              }
+            }
+          }
+        }
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&sm.full[s])) : "memory");
+      }
+      (void)kBX;
+    } else if (warp == 0) {
       // ------------------------------------------------------------ producer
       if (lane == 0) {
         for (uint32_t i = 0;; ++i) {
@@ -296,7 +401,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           const uint64_t ne = min(uint64_t(kTileElems), a.n - e0);
           const uint32_t bytes = uint32_t(ne * 4);
           const uint32_t tma_bytes = bytes & ~15u;
-          for (uint32_t k = tma_bytes / 4; k < ne; ++k) sm.in[s][k] = a.in[e0 + k];   // <= 3 tail floats
+          for (uint32_t k = tma_bytes / 4; k < ne; ++k) sm.in[s][k] = a.in[e0 + k];   // <= 3 tail floats  // sync: mbarrier full[s] (the producer's arrive.expect_tx releases them)
           mbar_arrive_expect_tx(&sm.full[s], tma_bytes);
           if (tma_bytes) tma_load_1d(sm.in[s], a.in + e0, tma_bytes, &sm.full[s]);
         }
@@ -325,7 +430,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         const uint64_t excl = resolve_excl(a.status, t, epoch, &nw, &ns);
         mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
         const TileMeta& md = sm.meta[m];
-        const uint32_t agg = md.agg;
+        const uint32_t agg = md.agg;  // sync: mbarrier staged[m]
         if (lane == 0 && t > 0) publish_prefix(a.status, t, excl + agg, epoch);
         {
           // F bytes of the tile (Fig 12 part 1): lane L converts group L's word
@@ -393,7 +498,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       const int w = warp - kFirstCompute;
       const Xpose xpose(lane);
       // scaled-float Lorenzo (quantize_scaled2) for the paper's default L = 32, order 1
-      constexpr bool kScaled = (M == 1 && O == 1);
+      constexpr bool kScaled = (M == 1 && O == 1 && D == 1);
       const float kf = lane ? -1.0f : -0.0f;
       const uint64_t nk = (uint64_t(__float_as_uint(kf)) << 32) | __float_as_uint(kf);
       uint32_t head = 0;                                // words this warp has appended (monotonic)
@@ -417,13 +522,13 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         if (t == kSentinel) break;                    // the writers stop on the ticket ring
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kCBPW * 32;   // first element of the warp
         float* src = &sm.in[s][w * kCBPW * 32];
-        if (t == a.num_tiles - 1) {
+        if (D == 1 && t == a.num_tiles - 1) {
           // virtual zero pad (R8): the ragged part of the last tile is zeroed in
           // shared memory once, so the encode loop needs no per-element test.
           // (No TMA writes this stage again in this launch: the producer's next
           // ticket is a sentinel; the proxy fence orders it anyway.)
           for (int k = lane; k < kCBPW * 32; k += 32)
-            if (g0 + k >= a.n) src[k] = 0.0f;
+            if (g0 + k >= a.n) src[k] = 0.0f;  // sync: own slice of the stage; no TMA rewrites it in this launch
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           __syncwarp();
         }
@@ -446,7 +551,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           float x[4];
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
-            x[q] = src[(4 * g + q) * 32 + lane];
+            x[q] = src[(4 * g + q) * 32 + lane];  // sync: mbarrier full[s] (TMA / cp.async / producer stores); stage reused after empty[s]
           }
           uint32_t r[4];
           float resmax = 0.0f;
@@ -481,7 +586,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           auto lorenzo_and_counts = [&]() {
             if constexpr (M == 1) {
 #pragma unroll
-              for (int q = 0; q < 4; ++q) v[q] = (O == 2) ? lorenzo2_pack(r[q], lane) : lorenzo_pack(r[q], lane);
+              for (int q = 0; q < 4; ++q)
+                v[q] = (D > 1) ? lorenzo_md_pack<D>(r[q], lane) : (O == 2) ? lorenzo2_pack(r[q], lane) : lorenzo_pack(r[q], lane);
             } else {
               // a block continues across its sub-blocks: lane 0 of sub-block q
               // takes lane 31 of sub-block q-1 unless q starts a block
@@ -595,8 +701,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               agg += *reinterpret_cast<volatile uint16_t*>(&md.cnt[k]);  // sync: atom.acq_rel on meta_done[m] (the last warp acquires every warp's count)
             publish_aggregate(a.status, t, agg, epoch);
             trace_put(a.trace, t, 2, global_ns());
-            md.tile = t;
-            md.agg = agg;
+            md.tile = t;  // sync: the last warp, then mbarrier staged[m]
+            md.agg = agg;  // sync: the last warp, then mbarrier staged[m]; slot reused after released
             sm.meta_done[m] = 0;
             mbar_arrive(&sm.staged[m]);
           }
@@ -609,7 +715,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   // R5 guard: some |r0| >= 2^22 (NaN and Inf included)
   uint32_t flag = 0;
   if (!eb_ok) flag = (a.n > 0) ? kBadRange : 0u;
-  else if (!(vmax < (O == 2 ? 0.5f * kGuard : kGuard)) || wmax > uint32_t(kMaxBlockWords)) flag = kBadRange;   // R5 / R17
+  else if (!(vmax < (O == 2 || D == 2 ? 0.5f * kGuard : D == 3 ? 0.25f * kGuard : kGuard)) ||
+           wmax > uint32_t(kMaxBlockWords))
+    flag = kBadRange;   // R5 / R17 / R18
 
   if (cta_finish(a.ws, flag)) {
     uint32_t final_status = CUSZP_OK;
@@ -623,7 +731,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       uint8_t* h = a.out;                                   // header (R10)
       *reinterpret_cast<uint32_t*>(h) = 0x505A5343u;        // "CSZP"
       h[4] = CUSZP_VERSION;
-      h[5] = uint8_t(a.mode | (O == 2 ? 0x10 : 0));        // predictor order (R17)
+      h[5] = uint8_t(a.mode | (O == 2 ? 0x10 : 0) | ((D - 1) << 5));   // predictor order (R17), dims (R18)
       h[6] = uint8_t(final_status);
       h[7] = uint8_t(5 + (M == 2 ? 1 : M == 4 ? 2 : 0));   // log2(L)
       *reinterpret_cast<uint64_t*>(h + 8) = a.n;
@@ -639,18 +747,20 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 }
 
 namespace {
-template <int M, int O = 1>
+template <int M, int O = 1, int D = 1>
 cudaError_t configure_m(int* occ) {
   const int smem = int(sizeof(CompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M, O>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M, O>, kCThreads, smem);
+  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M, O, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M, O, D>, kCThreads, smem);
   return e;
 }
 }  // namespace
 
 cudaError_t compress_configure(int M, int* occ) {
   int occ2 = 0;
-  if (M == 1 && configure_m<1, 2>(&occ2) != cudaSuccess) return cudaErrorUnknown;
+  if (M == 1 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
+                 configure_m<1, 1, 3>(&occ2) != cudaSuccess))
+    return cudaErrorUnknown;
   return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
 }
 
@@ -665,6 +775,8 @@ cudaError_t compress_launch(int M, int order, unsigned grid, const CompressArgs&
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  if (a.dims == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1, 2>, a);
+  if (a.dims == 3) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1, 3>, a);
   if (order == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 2>, a);
   if (M == 1) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1>, a);
   if (M == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<2, 1>, a);

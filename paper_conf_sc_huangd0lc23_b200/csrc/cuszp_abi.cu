@@ -75,20 +75,48 @@ uint32_t status_capacity(size_t ws_bytes) {
   return c > 0xffffffffull ? 0xffffffffu : uint32_t(c);
 }
 
+// Multi-dimensional Lorenzo (R18): block box and block grid of a field.
+struct MdGrid {
+  int dims = 1;
+  uint64_t nz = 1, ny = 1, nx = 0, nbz = 0, nby = 0, nbx = 0, nb = 0;
+};
+bool md_grid(size_t nz, size_t ny, size_t nx, int dims, MdGrid* g) {
+  if ((dims != 2 && dims != 3) || nz == 0 || ny == 0 || nx == 0) return false;
+  g->dims = dims;
+  g->nz = nz; g->ny = ny; g->nx = nx;
+  const uint64_t bz = dims == 3 ? 2 : 1, bx = dims == 3 ? 4 : 8;
+  g->nbz = (nz + bz - 1) / bz;
+  g->nby = (ny + 3) / 4;
+  g->nbx = (nx + bx - 1) / bx;
+  g->nb = g->nbz * g->nby * g->nbx;
+  return g->nb < (uint64_t(1) << 32) && nz * ny * nx / nz / ny == nx;   // 32-bit block ids; no overflow
+}
+
 int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const float* d_minmax,
                     int n_pairs, void* d_out, size_t out_capacity, unsigned long long* d_out_bytes,
-                    void* d_ws, size_t ws_bytes, cudaStream_t stream, int L = kL, int order = 1) {
+                    void* d_ws, size_t ws_bytes, cudaStream_t stream, int L = kL, int order = 1,
+                    const MdGrid* md = nullptr) {
   const int M = sub_blocks(L);
   if (!valid_L(L) || (order != 1 && order != 2) || (order == 2 && M != 1)) return CUSZP_EINVAL;
-  if (out_capacity < cuszp_max_compressed_bytes_L(n, L) || ws_bytes < cuszp_workspace_bytes(n))
+  const uint64_t nb = md ? md->nb : num_blocks(n, L);
+  // tiles of 128 blocks of 32 elements (4096 elements; M sub-blocks per L-block)
+  const uint64_t tiles = md ? (nb + kTileBlocks - 1) / kTileBlocks : num_tiles(n);
+  if (out_capacity < (md ? size_t(kHdr + align16(nb) + 128 * nb) : cuszp_max_compressed_bytes_L(n, L)) ||
+      ws_bytes < kWsCtrlBytes + 8 * (tiles > 0 ? tiles : 1))
     return CUSZP_ENOSPACE;
   DeviceInfo di;
   if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
   CompressArgs a;
   a.in = d_in;
   a.n = n;
-  a.nb = num_blocks(n, L);
-  a.num_tiles = uint32_t(num_tiles(n));
+  a.nb = nb;
+  a.num_tiles = uint32_t(tiles);
+  a.dims = md ? md->dims : 1;
+  a.nz = md ? md->nz : 1;
+  a.ny = md ? md->ny : 1;
+  a.nx = md ? md->nx : n;
+  a.nby = md ? md->nby : 1;
+  a.nbx = md ? md->nbx : nb;
   a.mode = mode;
   a.eb_in = eb_in;
   a.minmax = d_minmax;
@@ -268,6 +296,11 @@ int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t 
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
   a.trace = g_trace;
+  a.dims = 1;
+  a.nz = a.ny = 1;
+  a.nx = n;
+  a.nby = 1;
+  a.nbx = a.nb;
   if (small_L(block_len))
     return decompress_small_launch(block_len, a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK
                                                                                                 : CUSZP_ECUDA;
@@ -278,6 +311,88 @@ int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t 
   if (grid < 1) grid = 1;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   return decompress_launch(M, order, unsigned(grid), a, s) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+}
+
+size_t cuszp_num_blocks_md(size_t nz, size_t ny, size_t nx, int dims) {
+  MdGrid g;
+  return md_grid(nz, ny, nx, dims, &g) ? size_t(g.nb) : 0;
+}
+
+size_t cuszp_max_compressed_bytes_md(size_t nz, size_t ny, size_t nx, int dims) {
+  MdGrid g;
+  if (!md_grid(nz, ny, nx, dims, &g)) return 0;
+  return size_t(kHdr + align16(g.nb) + 128 * g.nb);   // 32-word garbage bound, as cuszp_max_compressed_bytes
+}
+
+size_t cuszp_workspace_bytes_md(size_t nz, size_t ny, size_t nx, int dims) {
+  MdGrid g;
+  if (!md_grid(nz, ny, nx, dims, &g)) return 0;
+  const uint64_t t = (g.nb + kTileBlocks - 1) / kTileBlocks;
+  return size_t(kWsCtrlBytes + 8 * (t > 0 ? t : 1));
+}
+
+int cuszp_compress_md(const float* d_in, size_t nz, size_t ny, size_t nx, int dims, float eb, int mode, void* d_out,
+                      size_t out_capacity, unsigned long long* d_out_bytes, void* d_ws, size_t ws_bytes,
+                      void* stream) {
+  MdGrid g;
+  if (d_in == nullptr || d_out == nullptr || d_ws == nullptr || !md_grid(nz, ny, nx, dims, &g)) return CUSZP_EINVAL;
+  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
+      (reinterpret_cast<uintptr_t>(d_ws) & 15u))
+    return CUSZP_EINVAL;
+  const size_t n = nz * ny * nx;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (out_capacity < cuszp_max_compressed_bytes_md(nz, ny, nx, dims) ||
+      ws_bytes < cuszp_workspace_bytes_md(nz, ny, nx, dims))
+    return CUSZP_ENOSPACE;
+  if (mode == CUSZP_ABS) {
+    if (!eb_is_normal(eb)) return CUSZP_EINVAL;
+    return launch_compress(d_in, n, CUSZP_ABS, eb, nullptr, 0, d_out, out_capacity, d_out_bytes, d_ws, ws_bytes, s,
+                           kL, 1, &g);
+  }
+  if (mode == CUSZP_REL) {
+    if (!(eb > 0.0f) || !(eb - eb == 0.0f)) return CUSZP_EINVAL;
+    const int st = cuszp_range(d_in, n, nullptr, d_ws, ws_bytes, stream);
+    if (st != CUSZP_OK) return st;
+    return launch_compress(d_in, n, CUSZP_REL, eb, static_cast<const WsCtrl*>(d_ws)->minmax, 1, d_out,
+                           out_capacity, d_out_bytes, d_ws, ws_bytes, s, kL, 1, &g);
+  }
+  return CUSZP_EINVAL;
+}
+
+int cuszp_decompress_md(const void* d_in, size_t in_bytes, float* d_out, size_t nz, size_t ny, size_t nx, int dims,
+                        void* d_ws, size_t ws_bytes, void* stream) {
+  MdGrid g;
+  if (d_in == nullptr || d_out == nullptr || d_ws == nullptr || !md_grid(nz, ny, nx, dims, &g)) return CUSZP_EINVAL;
+  if ((reinterpret_cast<uintptr_t>(d_in) & 15u) || (reinterpret_cast<uintptr_t>(d_out) & 15u) ||
+      (reinterpret_cast<uintptr_t>(d_ws) & 15u))
+    return CUSZP_EINVAL;
+  if (ws_bytes < cuszp_workspace_bytes_md(nz, ny, nx, dims)) return CUSZP_ENOSPACE;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  DecompressArgs a;
+  a.in = static_cast<const uint8_t*>(d_in);
+  a.in_bytes = in_bytes;
+  a.out = d_out;
+  a.n = nz * ny * nx;
+  a.nb = g.nb;
+  a.num_tiles = uint32_t((g.nb + kTileBlocks - 1) / kTileBlocks);
+  a.ws = static_cast<WsCtrl*>(d_ws);
+  a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
+  a.status_cap = status_capacity(ws_bytes);
+  a.trace = g_trace;
+  a.dims = dims;
+  a.nz = g.nz;
+  a.ny = g.ny;
+  a.nx = g.nx;
+  a.nby = g.nby;
+  a.nbx = g.nbx;
+  const int occ = di.occ_d[0];
+  uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
+  if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);
+  if (grid > a.num_tiles) grid = a.num_tiles;
+  if (grid < 1) grid = 1;
+  return decompress_launch(1, 1, unsigned(grid), a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK
+                                                                                                    : CUSZP_ECUDA;
 }
 
 int cuszp_last_status(const void* d_ws, void* stream) {

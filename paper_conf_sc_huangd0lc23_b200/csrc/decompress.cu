@@ -73,8 +73,11 @@ static_assert(kBarFree0 + 2 <= 16, "named barriers");
 // M = L / 32: see compress.cu -- sub-block i of a block
 // finds its word k at M k + i of the block's payload, and the in-block
 // prefix sum (a11) runs over the block's M sub-blocks.
-template <int M, int O>
+// D = Lorenzo dimensions (R18): 2 / 3 invert the block-local predictor of
+// 1x4x8 / 2x4x4 blocks and scatter each block's rows into the (nz, ny, nx) field.
+template <int M, int O, int D = 1>
 __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kernel(DecompressArgs a) {
+  static_assert(D == 1 || (M == 1 && O == 1), "multi-dimensional Lorenzo with L = 32, order 1");
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
   static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
   constexpr uint32_t kLog2L = 5 + (M == 2 ? 1 : M == 4 ? 2 : 0);
@@ -99,7 +102,8 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     eb = *reinterpret_cast<const float*>(h + 16);
     const uint64_t pbytes = *reinterpret_cast<const uint64_t*>(h + 24);
     if (magic != 0x505A5343u || h[4] != CUSZP_VERSION || h[7] != kLog2L ||
-        ((h[5] & 0x10) != 0) != (O == 2))                   // predictor order (R17)
+        ((h[5] & 0x10) != 0) != (O == 2) ||                 // predictor order (R17)
+        ((h[5] >> 5) & 3) != D - 1)                          // predictor dimensions (R18)
       err = CUSZP_ECORRUPT;
     else if (h[6] != CUSZP_OK) err = (h[6] == CUSZP_ERANGE) ? CUSZP_ERANGE : CUSZP_ECORRUPT;
     else if (hn != a.n) err = CUSZP_EINVAL;
@@ -364,7 +368,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           __syncwarp();
           const uint4 raw = *reinterpret_cast<const uint4*>(&scratch[row + lane4]);
           constexpr int kSeg = (32 - 8 * M) << 8;                     // segment = the block's 8 M lanes
-          if (O == 1 && scaled_ok) {
+          if (D == 1 && O == 1 && scaled_ok) {
             // v = 2|l| + s rotated right by one is sign | |l|: the bits of the
             // subnormal float l * 2^-149 (the encoder's
             // quantize_scaled2 in reverse).  Every sum the inverse Lorenzo
@@ -426,6 +430,54 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             e1 = (v1 & 1u) ? -int(v1 >> 1) : int(v1 >> 1);
             e2 = (v2 & 1u) ? -int(v2 >> 1) : int(v2 >> 1);
             e3 = (v3 & 1u) ? -int(v3 >> 1) : int(v3 >> 1);
+          }
+          if constexpr (D > 1) {
+            // R18: r = cumulative sums of l along x, y (and z) of the block.
+            // This lane holds elements 4 k8 .. 4 k8 + 3 of block q: 2D row
+            // k8/2, x = 4 (k8 % 2) + e; 3D plane k8/4, row k8 % 4, x = e.
+            const uint32_t k8 = lane & 7u;
+            constexpr int kSeg8 = 24 << 8, kSeg4 = 28 << 8;
+            e1 += e0;                                                 // along x, inside the lane
+            e2 += e1;
+            e3 += e2;
+            if constexpr (D == 2) {
+              const int cx = __shfl_up_sync(kFull, e3, 1);            // the row's left half
+              if (k8 & 1u) { e0 += cx; e1 += cx; e2 += cx; e3 += cx; }
+              e0 = scan_step_up(e0, 2, kSeg8); e1 = scan_step_up(e1, 2, kSeg8);   // along y (lanes 2 apart)
+              e2 = scan_step_up(e2, 2, kSeg8); e3 = scan_step_up(e3, 2, kSeg8);
+              e0 = scan_step_up(e0, 4, kSeg8); e1 = scan_step_up(e1, 4, kSeg8);
+              e2 = scan_step_up(e2, 4, kSeg8); e3 = scan_step_up(e3, 4, kSeg8);
+            } else {
+              e0 = scan_step_up(e0, 1, kSeg4); e1 = scan_step_up(e1, 1, kSeg4);   // along y (4-lane planes)
+              e2 = scan_step_up(e2, 1, kSeg4); e3 = scan_step_up(e3, 1, kSeg4);
+              e0 = scan_step_up(e0, 2, kSeg4); e1 = scan_step_up(e1, 2, kSeg4);
+              e2 = scan_step_up(e2, 2, kSeg4); e3 = scan_step_up(e3, 2, kSeg4);
+              e0 = scan_step_up(e0, 4, kSeg8); e1 = scan_step_up(e1, 4, kSeg8);   // along z
+              e2 = scan_step_up(e2, 4, kSeg8); e3 = scan_step_up(e3, 4, kSeg8);
+            }
+            float dd[4];
+            dd[0] = __fmul_rn(__int2float_rn(e0), two_eb);           // a12 (R13)
+            dd[1] = __fmul_rn(__int2float_rn(e1), two_eb);
+            dd[2] = __fmul_rn(__int2float_rn(e2), two_eb);
+            dd[3] = __fmul_rn(__int2float_rn(e3), two_eb);
+            const uint32_t b = t * uint32_t(kTileBlocks) + uint32_t(w) * kBPW + uint32_t(g) * 4u + q;
+            const uint32_t kx = b % uint32_t(a.nbx), kyz = b / uint32_t(a.nbx);
+            const uint32_t ky = kyz % uint32_t(a.nby), kz = kyz / uint32_t(a.nby);
+            uint64_t gz, gy, gx;
+            if constexpr (D == 2) { gz = kz; gy = ky * 4u + (k8 >> 1); gx = kx * 8u + 4u * (k8 & 1u); }
+            else { gz = kz * 2u + (k8 >> 2); gy = ky * 4u + (k8 & 3u); gx = kx * 4u; }
+            if (b < a.nb && gz < a.nz && gy < a.ny) {
+              float* o = a.out + (gz * a.ny + gy) * a.nx + gx;
+              if (gx + 4 <= a.nx && (reinterpret_cast<uintptr_t>(o) & 15u) == 0) {
+                *reinterpret_cast<float4*>(o) = make_float4(dd[0], dd[1], dd[2], dd[3]);
+              } else {
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                  if (gx + e < a.nx) o[e] = dd[e];
+              }
+            }
+            __syncwarp();
+            continue;
           }
           // a11: r_j = sum_{i <= j} l_i within the block
           e1 += e0;
@@ -498,18 +550,20 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 }
 
 namespace {
-template <int M, int O = 1>
+template <int M, int O = 1, int D = 1>
 cudaError_t configure_m(int* occ) {
   const int smem = int(sizeof(DecompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O>, kDThreads, smem);
+  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O, D>, kDThreads, smem);
   return e;
 }
 }  // namespace
 
 cudaError_t decompress_configure(int M, int* occ) {
   int occ2 = 0;
-  if (M == 1 && configure_m<1, 2>(&occ2) != cudaSuccess) return cudaErrorUnknown;
+  if (M == 1 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
+                 configure_m<1, 1, 3>(&occ2) != cudaSuccess))
+    return cudaErrorUnknown;
   return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
 }
 
@@ -524,6 +578,8 @@ cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressA
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  if (a.dims == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 2>, a);
+  if (a.dims == 3) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 3>, a);
   if (order == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 2>, a);
   if (M == 1) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1>, a);
   if (M == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<2, 1>, a);

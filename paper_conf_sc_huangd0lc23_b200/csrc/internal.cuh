@@ -427,6 +427,9 @@ struct CompressArgs {
   uint64_t* status;
   uint32_t status_cap;
   uint64_t* trace;           // diagnostics only (nullptr): 8 u64 per tile, see tools/trace_scan.py
+  int dims;                  // Lorenzo dimensions (R18): 1, or 2 / 3 over the (nz, ny, nx) field below
+  uint64_t nz, ny, nx;       // field shape (dims > 1; n = nz ny nx)
+  uint64_t nby, nbx;         // block grid rows / columns (dims > 1; nb = nbz nby nbx)
 };
 
 struct DecompressArgs {
@@ -440,6 +443,9 @@ struct DecompressArgs {
   uint64_t* status;
   uint32_t status_cap;
   uint64_t* trace;
+  int dims;                  // as CompressArgs
+  uint64_t nz, ny, nx;
+  uint64_t nby, nbx;
 };
 
 struct RangeArgs {
