@@ -20,6 +20,8 @@
 //         3 local adds + a 3-step segmented shuffle scan,
 //     a12 dequantise d' = (float) r * 2eb (R13), 128-bit stores.
 // Every read is bounded by in_bytes (corrupt input -> async ECORRUPT).
+#include <type_traits>
+
 #include "internal.cuh"
 
 namespace cuszp {
@@ -295,7 +297,10 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
       const uint32_t sel_quad = 0x4440u + q;                        // PRMT: byte q, zero-extended
       const uint32_t sel_pair = (q & 1) ? 0x4432u : 0x4410u;        // PRMT: half q&1, zero-extended
       const uint32_t row_pair = (q >> 1) * 32u, row_single = q * 32u;
+      const uint32_t sel_b01 = hi ? 0x4441u : 0x4440u, sel_b23 = hi ? 0x4443u : 0x4442u;
       const uint32_t lane4 = 4u * k8;
+      auto compute_role = [&](auto scaled_tag) {
+      constexpr bool kScaledD = decltype(scaled_tag)::value;
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kDStages);
         mbar_wait(&sm.full[s], (i / kDStages) & 1u);          // tile's payload landed (suspending wait)
@@ -348,10 +353,10 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             sel = sel_quad;
             row = 0;
           } else if (mode == 1) {
-            const uint32_t w0 = wbytes & 0xffu, w1 = (wbytes >> 8) & 0xffu;
-            const uint32_t w2 = (wbytes >> 16) & 0xffu, w3 = wbytes >> 24;
-            const uint32_t x01 = k16 < (hi ? w1 : w0) ? gdata[(hi ? w0 : 0u) + k16] : 0u;
-            const uint32_t x23 = k16 < (hi ? w3 : w2) ? gdata[w0 + w1 + (hi ? w2 : 0u) + k16] : 0u;
+            // lanes 0-15 take blocks 0 / 2, lanes 16-31 blocks 1 / 3: word counts
+            // and exclusive word offsets by per-lane byte selects
+            const uint32_t x01 = k16 < __byte_perm(wbytes, 0, sel_b01) ? gdata[__byte_perm(pbytes, 0, sel_b01) + k16] : 0u;
+            const uint32_t x23 = k16 < __byte_perm(wbytes, 0, sel_b23) ? gdata[__byte_perm(pbytes, 0, sel_b23) + k16] : 0u;
             scratch[lane] = xpose(x01);
             scratch[32 + lane] = xpose(x23);
             sel = sel_pair;
@@ -368,7 +373,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           __syncwarp();
           const uint4 raw = *reinterpret_cast<const uint4*>(&scratch[row + lane4]);
           constexpr int kSeg = (32 - 8 * M) << 8;                     // segment = the block's 8 M lanes
-          if (D == 1 && O == 1 && scaled_ok) {
+          if constexpr (kScaledD) {
             // v = 2|l| + s rotated right by one is sign | |l|: the bits of the
             // subnormal float l * 2^-149 (the encoder's
             // quantize_scaled2 in reverse).  Every sum the inverse Lorenzo
@@ -531,6 +536,14 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           __syncwarp();
         }
         named_arrive(kBarEmpty0 + s, kBarCount);
+      }
+      };
+      // one branch for the whole launch, not one per group
+      if constexpr (D == 1 && O == 1) {
+        if (scaled_ok) compute_role(std::true_type{});
+        else compute_role(std::false_type{});
+      } else {
+        compute_role(std::false_type{});
       }
     }
   }
