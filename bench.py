@@ -696,7 +696,9 @@ def run_ours(args, rank, world, dev):
         "ms_per_step": d["ms_per_step"], "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": cfg, "fields": [f for f in fields if f] or None, "rel": rels,
-                   "n_elements": n_total // len(rels), "n_per_rank": [x.numel() for x in xs.values()],
+                   "n_elements": n_total // len(rels),
+                   "n_per_rank": [b - a for a, b in (slab(n_total // len(rels) // len(fields), p, world)
+                                                     for p in range(world))],
                    "round_trips_per_step": len(jobs),
                    "parallelism": f"sharded x{world} (block-aligned slabs, global range)" if world > 1 else "single",
                    "l2": "inputs > L2; flushed anyway (512 MB write + read, untimed) before every round trip"},

@@ -47,15 +47,33 @@ def slab_bounds(n_total: int, rank: int, world: int) -> tuple[int, int]:
     return min(b0 * BLOCK, n_total), min(b1 * BLOCK, n_total)
 
 
+def _nccl(group) -> bool:
+    return dist.get_backend(group) == "nccl"
+
+
 def _allgather(dst: torch.Tensor, src: torch.Tensor, group) -> torch.Tensor:
-    if dist.get_backend(group) == "nccl":
+    if _nccl(group):
         dist.all_gather_into_tensor(dst, src, group=group)
     else:
+        # gloo (CPU tests; several ranks sharing one GPU): host staging
         world = dist.get_world_size(group)
-        parts = list(dst.view(world, -1).unbind(0))
-        dist.all_gather(parts, src, group=group)
-        dst.copy_(torch.stack(parts).view(-1))
+        parts = [torch.empty_like(src, device="cpu") for _ in range(world)]
+        dist.all_gather(parts, src.cpu(), group=group)
+        dst.copy_(torch.cat(parts).view(-1))
     return dst
+
+
+def _broadcast(t: torch.Tensor, src: int, group) -> None:
+    if _nccl(group) or not t.is_cuda:
+        dist.broadcast(t, src=src, group=group)
+    else:
+        tmp = t.cpu()
+        dist.broadcast(tmp, src=src, group=group)
+        t.copy_(tmp)
+
+
+def _send(t: torch.Tensor, dst: int, group) -> None:
+    dist.send(t if (_nccl(group) or not t.is_cuda) else t.cpu(), dst=dst, group=group)
 
 
 def allgather_minmax(mm_local: torch.Tensor, mm_all: torch.Tensor, group=None) -> torch.Tensor:
@@ -196,8 +214,7 @@ def gather_container(res: ShardResult, group=None, dst: int | None = None) -> to
     mine = res.stream[: h["bytes"][rank]]
     if dst is not None and rank != dst:
         if h["bytes"][rank]:
-            dist.send(mine.contiguous(), dst=dist.get_global_rank(group, dst) if group is not None else dst,
-                      group=group)
+            _send(mine.contiguous(), dist.get_global_rank(group, dst) if group is not None else dst, group)
         return None
     buf = torch.zeros(total, dtype=torch.uint8, device=dev)
     buf[:base] = _header_bytes_tensor(res.header)
@@ -207,8 +224,8 @@ def gather_container(res: ShardResult, group=None, dst: int | None = None) -> to
         for p in range(world):
             if h["bytes"][p]:
                 src = dist.get_global_rank(group, p) if group is not None else p
-                dist.broadcast(views[p], src=src, group=group)
-    else:
+                _broadcast(views[p], src, group)
+    elif _nccl(group) or not buf.is_cuda:
         ops = []
         for p in range(world):
             if p != rank and h["bytes"][p]:
@@ -217,6 +234,13 @@ def gather_container(res: ShardResult, group=None, dst: int | None = None) -> to
         if ops:
             for w in dist.batch_isend_irecv(ops):
                 w.wait()
+    else:
+        for p in range(world):                               # gloo + CUDA buffers: host staging
+            if p != rank and h["bytes"][p]:
+                src = dist.get_global_rank(group, p) if group is not None else p
+                tmp = torch.empty(views[p].numel(), dtype=torch.uint8)
+                dist.recv(tmp, src=src, group=group)
+                views[p].copy_(tmp)
     return buf
 
 

@@ -1,6 +1,6 @@
 """Summarise the ncu evidence of one round into profiles/ (committed).
 
-    python tools/profile_summary.py <full.ncu-rep> <launches.csv> <round tag>
+    python tools/profile_summary.py <full.ncu-rep> <launches.csv> <round tag> [workload] [n_elements]
 
 Writes profiles/<tag>_ncu_summary.txt (per kernel: duration, DRAM bytes,
 throughput, issue/occupancy, top stalls), profiles/<tag>_launches_share.txt
@@ -39,11 +39,15 @@ def kname(s: str) -> str | None:
 
 def main():
     rep, launches, tag = sys.argv[1], sys.argv[2], sys.argv[3]
+    workload = sys.argv[4] if len(sys.argv) > 4 else None
+    n_el = int(sys.argv[5]) if len(sys.argv) > 5 else None
     os.makedirs(OUT, exist_ok=True)
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
     lines, js = [], {"dram_bytes_per_launch": {}, "source": os.path.basename(rep), "tag": tag}
+    if workload:
+        js["workload"] = workload
     for r in rows[2:]:
         k = kname(r[hdr.index("Kernel Name")])
         if k is None:
@@ -70,6 +74,10 @@ def main():
         dur = float(vals["gpu__time_duration.sum"][0]) * {"usecond": 1e-6, "msecond": 1e-3, "nsecond": 1e-9}.get(
             vals["gpu__time_duration.sum"][1].lower(), 1e-6)
         lines.append(f"   => DRAM traffic {tb / 1e6:.2f} MB per launch, {tb / dur / 1e9:.1f} GB/s over the launch")
+        if n_el and "smsp__inst_executed.sum" in vals:
+            ipb = float(vals["smsp__inst_executed.sum"][0]) / ((n_el + 31) // 32)
+            lines.append(f"   => {ipb:.1f} warp instructions per 32-element block")
+            js.setdefault("warp_inst_per_block", {})[k] = round(ipb, 2)
         js["dram_bytes_per_launch"].setdefault(k, tb)
     with open(os.path.join(OUT, f"{tag}_ncu_summary.txt"), "w") as f:
         f.write("\n".join(lines) + "\n")
