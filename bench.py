@@ -419,17 +419,23 @@ def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int)
     length), brings it back, decompresses and D2H-copies the reconstruction;
     consecutive jobs rotate over streams so one job's device->host traffic
     overlaps the next one's host->device traffic.  Wall clock, max over ranks."""
-    n_lanes = int(os.environ.get("CUSZP_E2E_LANES", "2" if nmax > (1 << 27) else "3"))
-    lanes = []
-    for _ in range(n_lanes):
-        lanes.append(dict(stream=torch.cuda.Stream(dev),
-                          h_out=torch.zeros(cap, dtype=torch.uint8).pin_memory(),
-                          h_len=torch.zeros(1, dtype=torch.int64).pin_memory(),
-                          h_y=torch.empty(nmax, dtype=torch.float32).pin_memory(),
-                          d_in=torch.empty(nmax, dtype=torch.float32, device=dev),
-                          d_out=torch.empty(cap, dtype=torch.uint8, device=dev),
-                          d_y=torch.empty(nmax, dtype=torch.float32, device=dev),
-                          ws=cz.Workspace(nmax, dev)))
+    # Compressions run on "C" streams (host->device heavy: the field in, the
+    # stream out) and decompressions on "D" streams (the stream in, the field
+    # out), each job's decompression event-ordered after its compression, so
+    # the two directions of the link carry balanced traffic at all times.
+    n_sets = int(os.environ.get("CUSZP_E2E_LANES", "2"))
+    sets = []
+    for _ in range(n_sets):
+        sets.append(dict(cs=torch.cuda.Stream(dev), ds=torch.cuda.Stream(dev),
+                         h_out=torch.zeros(cap, dtype=torch.uint8).pin_memory(),
+                         h_len=torch.zeros(1, dtype=torch.int64).pin_memory(),
+                         h_y=torch.empty(nmax, dtype=torch.float32).pin_memory(),
+                         d_in=torch.empty(nmax, dtype=torch.float32, device=dev),
+                         d_out=torch.empty(cap, dtype=torch.uint8, device=dev),
+                         d_sin=torch.empty(cap, dtype=torch.uint8, device=dev),
+                         d_y=torch.empty(nmax, dtype=torch.float32, device=dev),
+                         wsc=cz.Workspace(nmax, dev), wsd=cz.Workspace(nmax, dev),
+                         comp_done=torch.cuda.Event(), dec_done=torch.cuda.Event(), used=False))
     lens = {}
     k = 0
     for i in range(1 + steps):
@@ -439,16 +445,23 @@ def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int)
                 torch.distributed.barrier()
             t0 = time.perf_counter()
         for lab, h_in, rel in jobs_host:
-            ln = lanes[k % n_lanes]
+            st = sets[k % n_sets]
             k += 1
             n = h_in.numel()
-            cz.compress_host_async(h_in, rel, "rel", ln["h_out"], ln["h_len"], ln["d_in"][:n], ln["d_out"],
-                                   ln["ws"], stream=ln["stream"])
-            cz.decompress_host_async(ln["h_out"], ln["h_y"][:n], ln["d_out"], ln["d_y"][:n], ln["ws"],
-                                     stream=ln["stream"])
+            if st["used"]:
+                st["cs"].wait_event(st["dec_done"])          # h_out is free once the last decompression read it
+            cz.compress_host_async(h_in, rel, "rel", st["h_out"], st["h_len"], st["d_in"][:n], st["d_out"],
+                                   st["wsc"], stream=st["cs"])
+            st["comp_done"].record(st["cs"])
+            st["ds"].wait_event(st["comp_done"])
+            cz.decompress_host_async(st["h_out"], st["h_y"][:n], st["d_sin"], st["d_y"][:n], st["wsd"],
+                                     stream=st["ds"])
+            st["dec_done"].record(st["ds"])
+            st["used"] = True
             if i == 0:      # warm-up pass: record the stream lengths (bytes counted per step)
-                ln["stream"].synchronize()
-                lens[lab] = int(ln["h_len"].item())
+                st["ds"].synchronize()
+                lens[lab] = int(st["h_len"].item())
+    n_lanes = 2 * n_sets
     torch.cuda.synchronize(dev)
     t_e2e = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
     if world > 1:
@@ -460,12 +473,12 @@ def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int)
         d2h += lens[lab] + 8 + 4 * n          # stream + its length out, reconstruction out
     # the last job's reconstruction in host memory satisfies the bound
     lab, h_in, rel = jobs_host[-1]
-    ln = lanes[(k - 1) % n_lanes]
+    ln = sets[(k - 1) % n_sets]
     n = h_in.numel()
     eb_l = float(np.frombuffer(ln["h_out"][16:20].numpy().tobytes(), np.float32)[0])
     err = (ln["h_y"][:n].double() - h_in.double()).abs().max().item()
     assert err <= eb_l + float(np.spacing(np.float32(h_in.abs().max().item()))), (err, eb_l)
-    del lanes
+    del sets
     # the host link's own ceiling for this traffic: both directions at once (copy engines)
     s1, s2 = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
     pa = torch.empty(1 << 28, dtype=torch.uint8).pin_memory()
@@ -491,8 +504,8 @@ def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int)
     return {"value": in_step * steps * world / float(t_e2e.item()) / 1e9, "unit": "GB/s",
             "link_gbs_per_direction": round(link_gbs, 1), "link_bound_gbs": round(bound, 1),
             "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-            "path": "cuszp_compress_host_async + cuszp_decompress_host_async (pinned host buffers, "
-                    f"{n_lanes} streams, wall clock)"}
+            "path": "cuszp_compress_host_async + cuszp_decompress_host_async (pinned host buffers; "
+                    f"compressions and decompressions on {n_lanes} streams, event-ordered; wall clock)"}
 
 
 def graph_replay_c1(r: Runner, steps: int, peak: float) -> dict:
