@@ -70,6 +70,12 @@ uint64_t* g_trace = nullptr;
 // occupancy-derived default); used by the look-back stress tests.
 int g_grid_compress = 0, g_grid_decompress = 0;
 
+// Decompression look-back chunk: 8 tiles once every CTA of the persistent
+// grid gets >= 24 tiles (the scanner's per-chunk latency then hides behind
+// the decode; measured -13 % on the 1.1 GB field), else 4 (balance on small
+// inputs: 8-tile chunks cost +5..15 % at 100 MB).  DESIGN sec 8.1.
+uint32_t decompress_chunk_tiles(uint64_t tiles, uint64_t grid) { return tiles >= 24 * grid ? 8u : 4u; }
+
 uint32_t status_capacity(size_t ws_bytes) {
   const uint64_t c = (ws_bytes - kWsCtrlBytes) / 8;
   return c > 0xffffffffull ? 0xffffffffu : uint32_t(c);
@@ -307,6 +313,7 @@ int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t 
   const int occ = di.occ_d[mi(M)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);
+  a.chunk_tiles = decompress_chunk_tiles(a.num_tiles, grid);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -389,6 +396,7 @@ int cuszp_decompress_md(const void* d_in, size_t in_bytes, float* d_out, size_t 
   const int occ = di.occ_d[0];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);
+  a.chunk_tiles = decompress_chunk_tiles(a.num_tiles, grid);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   return decompress_launch(1, 1, unsigned(grid), a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK

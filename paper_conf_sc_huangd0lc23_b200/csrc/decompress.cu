@@ -39,7 +39,14 @@ constexpr int kDStages = CUSZP_D_STAGES;
 #define CUSZP_D_UNROLL 4
 #endif
 constexpr int kDUnroll = CUSZP_D_UNROLL;                        // decode groups interleaved per iteration
-constexpr int kChunkTiles = 4;                                  // tiles per look-back unit
+#ifndef CUSZP_D_CHUNK_TILES
+#define CUSZP_D_CHUNK_TILES 8
+#endif
+// tiles per look-back unit: the scanner's latency per chunk (F loads + one
+// look-back, ~2 + ~7 us under load) must stay below the CTA's decode time of
+// the chunk (~1.8 us per tile), else the loader starves
+constexpr int kChunkTiles = CUSZP_D_CHUNK_TILES;
+static_assert(kChunkTiles == 4 || kChunkTiles == 8, "chunk of 4 or 8 tiles");
 constexpr int kGroups = kTileBlocks / 4;                        // 32 decode groups per tile
 constexpr int kDataWords = kTileBlocks * kMaxBlockWords + 8;   // 3208 words: worst tile + alignment slack
 constexpr int kDFirstCompute = 2;
@@ -77,8 +84,11 @@ static_assert(kBarFree0 + 2 <= 16, "named barriers");
 // prefix sum (a11) runs over the block's M sub-blocks.
 // D = Lorenzo dimensions (R18): 2 / 3 invert the block-local predictor of
 // 1x4x8 / 2x4x4 blocks and scatter each block's rows into the (nz, ny, nx) field.
-template <int M, int O, int D = 1>
+// CT = tiles per look-back chunk (4 or 8; 8 is instantiated for the main path
+// only, chosen by the host for large inputs).
+template <int M, int O, int D = 1, int CT = 4>
 __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kernel(DecompressArgs a) {
+  static_assert(CT == 4 || CT == 8, "chunk of 4 or 8 tiles");
   static_assert(D == 1 || (M == 1 && O == 1), "multi-dimensional Lorenzo with L = 32, order 1");
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
   static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
@@ -117,7 +127,8 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     }
   }
   const float two_eb = __fadd_rn(eb, eb);
-  const uint32_t num_chunks = (a.num_tiles + kChunkTiles - 1) / kChunkTiles;
+  constexpr uint32_t ct = CT;
+  const uint32_t num_chunks = (a.num_tiles + ct - 1) / ct;
   uint32_t bad = 0;
 
   if (threadIdx.x == 0) {
@@ -144,82 +155,110 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           named_arrive(kBarReady0 + b, 64);
           break;
         }
-        const uint32_t t0 = c * kChunkTiles;
-        const uint32_t ntiles = min(uint32_t(kChunkTiles), a.num_tiles - t0);
-        // lane L: sub-blocks 16L .. 16L+15 of the chunk = groups 4(L%8) .. +3 of
-        // tile L/8 = blocks (16L .. 16L+15) / M
-        const uint64_t blk = (uint64_t(t0) * kTileBlocks + 16u * lane) / M;
-        uint32_t fw[4] = {0, 0, 0, 0};
-        if (blk < a.nb) {                                              // in the 16-B padded F area
-          if constexpr (M == 1) {
-            const uint4 fq = *reinterpret_cast<const uint4*>(a.in + kHdr + blk);
-            fw[0] = fq.x; fw[1] = fq.y; fw[2] = fq.z; fw[3] = fq.w;
-          } else if constexpr (M == 2) {
-            // F of blocks 2g, 2g+1 replicated onto sub-blocks (4g .. 4g+3)
-            const uint2 fq = *reinterpret_cast<const uint2*>(a.in + kHdr + blk);
-            fw[0] = __byte_perm(fq.x, 0, 0x1100u); fw[1] = __byte_perm(fq.x, 0, 0x3322u);
-            fw[2] = __byte_perm(fq.y, 0, 0x1100u); fw[3] = __byte_perm(fq.y, 0, 0x3322u);
-          } else {
-            const uint32_t fq = *reinterpret_cast<const uint32_t*>(a.in + kHdr + blk);
-            fw[0] = __byte_perm(fq, 0, 0x0000u); fw[1] = __byte_perm(fq, 0, 0x1111u);
-            fw[2] = __byte_perm(fq, 0, 0x2222u); fw[3] = __byte_perm(fq, 0, 0x3333u);
+        const uint32_t t0 = c * ct;
+        const uint32_t ntiles = min(ct, a.num_tiles - t0);
+#ifdef CUSZP_TRACE
+        if (a.trace && uint32_t(lane) < ntiles) trace_put(a.trace, t0 + lane, 0, global_ns());
+#endif
+        // The chunk in parts of 4 tiles (ct / 4 of them): in part h, lane L takes
+        // sub-blocks 16L .. 16L+15 of tiles 4h .. 4h+3 = groups 4(L%8) .. +3 of
+        // tile 4h + L/8 = blocks (16L ..)/M.  All F loads of the chunk are
+        // issued before any is used (one memory latency per chunk).
+        constexpr int kParts = CT / 4;
+        uint32_t fw[kParts][4];
+        uint64_t blkp[kParts];
+#pragma unroll
+        for (int h = 0; h < kParts; ++h) {
+          const uint64_t blk = (uint64_t(t0 + 4 * h) * kTileBlocks + 16u * lane) / M;
+          blkp[h] = blk;
+          fw[h][0] = fw[h][1] = fw[h][2] = fw[h][3] = 0;
+          if (blk < a.nb) {                                              // in the 16-B padded F area
+            if constexpr (M == 1) {
+              const uint4 fq = *reinterpret_cast<const uint4*>(a.in + kHdr + blk);
+              fw[h][0] = fq.x; fw[h][1] = fq.y; fw[h][2] = fq.z; fw[h][3] = fq.w;
+            } else if constexpr (M == 2) {
+              // F of blocks 2g, 2g+1 replicated onto sub-blocks (4g .. 4g+3)
+              const uint2 fq = *reinterpret_cast<const uint2*>(a.in + kHdr + blk);
+              fw[h][0] = __byte_perm(fq.x, 0, 0x1100u); fw[h][1] = __byte_perm(fq.x, 0, 0x3322u);
+              fw[h][2] = __byte_perm(fq.y, 0, 0x1100u); fw[h][3] = __byte_perm(fq.y, 0, 0x3322u);
+            } else {
+              const uint32_t fq = *reinterpret_cast<const uint32_t*>(a.in + kHdr + blk);
+              fw[h][0] = __byte_perm(fq, 0, 0x0000u); fw[h][1] = __byte_perm(fq, 0, 0x1111u);
+              fw[h][2] = __byte_perm(fq, 0, 0x2222u); fw[h][3] = __byte_perm(fq, 0, 0x3333u);
+            }
           }
         }
-        uint32_t gw[4], gspan[4], gsum[4], lsum = 0;
+        uint32_t ttot[CT], agg = 0, tpre[CT];
+        const int tl = lane >> 3;
 #pragma unroll
-        for (int g = 0; g < 4; ++g) {
-          gw[g] = 0;
-          gspan[g] = 0;
-          gsum[g] = 0;
+        for (int h = 0; h < kParts; ++h) {
+          const uint64_t blk = blkp[h];
+          uint32_t gw[4], gspan[4], gsum[4], lsum = 0;
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            gw[g] = 0;
+            gspan[g] = 0;
+            gsum[g] = 0;
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              uint32_t f = (fw[h][g] >> (8 * k)) & 0xffu;
+              if (blk + (4 * g + k) / M >= a.nb) f = 0;
+              if (f > uint32_t(kMaxF)) { bad |= kBadCorrupt; f = 0; }
+              const uint32_t wq = f ? f + 1 : 0;             // Eq 2 in 4-byte words
+              gw[g] |= wq << (8 * k);
+              gspan[g] = max(gspan[g], wq);
+              gsum[g] += wq;
+            }
+            lsum += gsum[g];
+          }
+          // tile-local exclusive offsets: segmented scan over the 8 lanes of each tile
+          uint32_t incl = lsum;
+          incl = uint32_t(scan_step_up(int(incl), 1, 24 << 8));
+          incl = uint32_t(scan_step_up(int(incl), 2, 24 << 8));
+          incl = uint32_t(scan_step_up(int(incl), 4, 24 << 8));
+          uint32_t off = incl - lsum;
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            const uint32_t mode = gspan[g] <= 8 ? 0u : (gspan[g] <= 16 ? 1u : 2u);
+            cd.gwords[4 * h + tl][4 * (lane & 7) + g] = gw[g];
+            cd.gmeta[4 * h + tl][4 * (lane & 7) + g] = off | (mode << 16);
+            off += gsum[g];
+          }
+          // tile totals and the chunk aggregate
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
-            uint32_t f = (fw[g] >> (8 * k)) & 0xffu;
-            if (blk + (4 * g + k) / M >= a.nb) f = 0;
-            if (f > uint32_t(kMaxF)) { bad |= kBadCorrupt; f = 0; }
-            const uint32_t wq = f ? f + 1 : 0;             // Eq 2 in 4-byte words
-            gw[g] |= wq << (8 * k);
-            gspan[g] = max(gspan[g], wq);
-            gsum[g] += wq;
+            ttot[4 * h + k] = __shfl_sync(kFull, incl, 8 * k + 7);
+            tpre[4 * h + k] = agg;
+            agg += ttot[4 * h + k];
           }
-          lsum += gsum[g];
-        }
-        // tile-local exclusive offsets: segmented scan over the 8 lanes of each tile
-        uint32_t incl = lsum;
-        incl = uint32_t(scan_step_up(int(incl), 1, 24 << 8));
-        incl = uint32_t(scan_step_up(int(incl), 2, 24 << 8));
-        incl = uint32_t(scan_step_up(int(incl), 4, 24 << 8));
-        const int tl = lane >> 3;
-        uint32_t off = incl - lsum;
-#pragma unroll
-        for (int g = 0; g < 4; ++g) {
-          const uint32_t mode = gspan[g] <= 8 ? 0u : (gspan[g] <= 16 ? 1u : 2u);
-          cd.gwords[tl][4 * (lane & 7) + g] = gw[g];
-          cd.gmeta[tl][4 * (lane & 7) + g] = off | (mode << 16);
-          off += gsum[g];
-        }
-        // tile totals and the chunk aggregate
-        uint32_t ttot[kChunkTiles], agg = 0, tpre[kChunkTiles];
-#pragma unroll
-        for (int k = 0; k < kChunkTiles; ++k) {
-          ttot[k] = __shfl_sync(kFull, incl, 8 * k + 7);
-          tpre[k] = agg;
-          agg += ttot[k];
         }
         // a9: global synchronisation (decoupled look-back over chunks)
         if (lane == 0) publish_aggregate(a.status, c, agg, epoch);
+#ifdef CUSZP_TRACE
+        if (a.trace && uint32_t(lane) < ntiles) trace_put(a.trace, t0 + lane, 1, global_ns());
+        uint32_t tr_nw = 0, tr_ns = 0;
+        const uint64_t excl = resolve_prefix(a.status, c, agg, epoch, &tr_nw, &tr_ns);
+        if (a.trace && uint32_t(lane) < ntiles) {
+          trace_put(a.trace, t0 + lane, 2, global_ns());
+          trace_put(a.trace, t0 + lane, 6, (uint64_t(tr_nw) << 32) | tr_ns);
+        }
+#else
         const uint64_t excl = resolve_prefix(a.status, c, agg, epoch);
+#endif
         const bool oob = excl + agg > payload_words;   // corrupt offsets: decode zeros, never read past in_bytes
         if (oob) {
           bad |= kBadCorrupt;
 #pragma unroll
-          for (int g = 0; g < 4; ++g) cd.gwords[tl][4 * (lane & 7) + g] = 0u;
+          for (int h = 0; h < kParts; ++h)
+#pragma unroll
+            for (int g = 0; g < 4; ++g) cd.gwords[4 * h + tl][4 * (lane & 7) + g] = 0u;
         }
         uint64_t ts = 0;
         uint32_t tw = 0;
 #pragma unroll
-        for (int k = 0; k < kChunkTiles; ++k)
+        for (int k = 0; k < CT; ++k)
           if (lane == k) { ts = excl + tpre[k]; tw = oob ? 0u : ttot[k]; }
-        if (lane < kChunkTiles) {
+        if (lane < CT) {
           cd.tile_start[lane] = ts;
           cd.tile_words[lane] = tw;
         }
@@ -270,10 +309,13 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           }
           __syncwarp();
           if (lane == 0) {
-            sm.tile[s] = cd.chunk * kChunkTiles + j;  // sync: mbarrier full[s]
+            sm.tile[s] = cd.chunk * ct + j;  // sync: mbarrier full[s]
             sm.delta[s] = delta;  // sync: mbarrier full[s]
             mbar_arrive_expect_tx(&sm.full[s], tma_bytes);   // one phase per use, even with 0 bytes
             if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
+#ifdef CUSZP_TRACE
+            trace_put(a.trace, cd.chunk * ct + j, 3, global_ns());
+#endif
           }
           ++k;
         }
@@ -306,6 +348,13 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
         mbar_wait(&sm.full[s], (i / kDStages) & 1u);          // tile's payload landed (suspending wait)
         const uint32_t t = sm.tile[s];  // sync: mbarrier full[s]
         if (t == kSentinel) break;
+#ifdef CUSZP_TRACE
+        if (a.trace && lane == 0) {
+          const uint64_t now = global_ns();
+          if (w == 0) trace_put(a.trace, t, 4, now);
+          a.trace[16ull * a.num_tiles + 8ull * t + w] = now;          // per-warp pickup time
+        }
+#endif
         const bool last = (t == a.num_tiles - 1);
         const uint32_t* data = sm.data[s] + sm.delta[s];  // sync: mbarrier full[s]
         float* outp = a.out + uint64_t(t) * kTileElems + uint64_t(w) * kBPW * 32 + q * 32u + lane4;
@@ -535,6 +584,13 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           }
           __syncwarp();
         }
+#ifdef CUSZP_TRACE
+        if (a.trace && lane == 0) {
+          const uint64_t now = global_ns();
+          a.trace[8ull * a.num_tiles + 8ull * t + w] = now;          // per-warp done time
+          atomicMax(reinterpret_cast<unsigned long long*>(a.trace + 8ull * t + 5), now);
+        }
+#endif
         named_arrive(kBarEmpty0 + s, kBarCount);
       }
       };
@@ -563,11 +619,11 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 }
 
 namespace {
-template <int M, int O = 1, int D = 1>
+template <int M, int O = 1, int D = 1, int CT = 4>
 cudaError_t configure_m(int* occ) {
   const int smem = int(sizeof(DecompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O, D>, kDThreads, smem);
+  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O, D, CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O, D, CT>, kDThreads, smem);
   return e;
 }
 }  // namespace
@@ -575,7 +631,7 @@ cudaError_t configure_m(int* occ) {
 cudaError_t decompress_configure(int M, int* occ) {
   int occ2 = 0;
   if (M == 1 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
-                 configure_m<1, 1, 3>(&occ2) != cudaSuccess))
+                 configure_m<1, 1, 3>(&occ2) != cudaSuccess || configure_m<1, 1, 1, 8>(&occ2) != cudaSuccess))
     return cudaErrorUnknown;
   return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
 }
@@ -594,6 +650,7 @@ cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressA
   if (a.dims == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 2>, a);
   if (a.dims == 3) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 3>, a);
   if (order == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 2>, a);
+  if (M == 1 && a.chunk_tiles == 8) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 1, 8>, a);
   if (M == 1) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1>, a);
   if (M == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<2, 1>, a);
   return cudaLaunchKernelEx(&cfg, decompress_kernel<4, 1>, a);

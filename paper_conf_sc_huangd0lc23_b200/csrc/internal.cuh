@@ -446,6 +446,7 @@ struct DecompressArgs {
   int dims;                  // as CompressArgs
   uint64_t nz, ny, nx;
   uint64_t nby, nbx;
+  uint32_t chunk_tiles;      // tiles per look-back chunk: 8 for large inputs, 4 for small ones (balance)
 };
 
 struct RangeArgs {

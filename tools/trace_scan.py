@@ -102,7 +102,7 @@ def main():
     ob = torch.zeros(1, dtype=torch.int64, device=dev)
     mm = torch.empty(2, dtype=torch.float32, device=dev)
     y = torch.empty(n, dtype=torch.float32, device=dev)
-    trace = torch.zeros(nt * 16, dtype=torch.int64, device=dev)
+    trace = torch.zeros(nt * 24, dtype=torch.int64, device=dev)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     sp = torch.cuda.current_stream().cuda_stream
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
@@ -126,7 +126,13 @@ def main():
         torch.cuda.synchronize()
     h.cuszp_debug_set_trace(None)
     trd = trace[: nt * 8].view(nt, 8).cpu().numpy().astype(np.int64)
-    pw = trace[nt * 8:].view(nt, 8).cpu().numpy().astype(np.int64)
+    pw = trace[nt * 8:nt * 16].view(nt, 8).cpu().numpy().astype(np.int64)
+    pk = trace[nt * 16:].view(nt, 8).cpu().numpy().astype(np.int64)
+    busy = (pw - pk) / 1e3
+    print("decompress per-warp tile compute (pickup -> done, us):", pct(busy.ravel()))
+    # per warp slot, consecutive tiles of the same CTA are not identifiable; use the
+    # distribution of each warp's pickup relative to the tile's TMA issue instead
+    wait = (pk - trd_issue[:, None]) / 1e3 if False else None
     last = np.argmax(pw, axis=1)
     spread = (pw.max(axis=1) - pw.min(axis=1)) / 1e3
     print("decompress: which compute warp finishes a tile last:", np.bincount(last, minlength=8).tolist(),
