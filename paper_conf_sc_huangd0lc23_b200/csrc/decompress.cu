@@ -315,6 +315,7 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
 #ifdef CUSZP_TRACE
             trace_put(a.trace, cd.chunk * ct + j, 3, global_ns());
+            trace_put(a.trace, cd.chunk * ct + j, 7, blockIdx.x);
 #endif
           }
           ++k;
@@ -490,7 +491,8 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             // This lane holds elements 4 k8 .. 4 k8 + 3 of block q: 2D row
             // k8/2, x = 4 (k8 % 2) + e; 3D plane k8/4, row k8 % 4, x = e.
             const uint32_t k8 = lane & 7u;
-            constexpr int kSeg8 = 24 << 8, kSeg4 = 28 << 8;
+            constexpr int kSeg8 = 24 << 8;
+            [[maybe_unused]] constexpr int kSeg4 = 28 << 8;
             e1 += e0;                                                 // along x, inside the lane
             e2 += e1;
             e3 += e2;

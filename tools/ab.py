@@ -18,6 +18,7 @@ def load(path):
     sz, vp, i32, f32 = C.c_size_t, C.c_void_p, C.c_int, C.c_float
     h.cuszp_range.argtypes = [vp, sz, vp, vp, sz, vp]
     h.cuszp_compress_minmax.argtypes = [vp, sz, f32, vp, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_compress.argtypes = [vp, sz, f32, i32, vp, sz, vp, vp, sz, vp]
     h.cuszp_decompress.argtypes = [vp, sz, vp, sz, vp, sz, vp]
     h.cuszp_workspace_bytes.argtypes = [sz]; h.cuszp_workspace_bytes.restype = sz
     h.cuszp_max_compressed_bytes.argtypes = [sz]; h.cuszp_max_compressed_bytes.restype = sz
@@ -60,8 +61,8 @@ def main():
                 sink.copy_(flush_buf.view(torch.int64).sum())
     flush = _F
     sp = torch.cuda.current_stream().cuda_stream
-    ev = [torch.cuda.Event(enable_timing=True) for _ in range(9)]
-    res = {i: {"range": [], "compress": [], "decompress": [], "rel_chain": []} for i in range(len(libs))}
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(11)]
+    res = {i: {"range": [], "compress": [], "decompress": [], "rel_chain": [], "rel_call": []} for i in range(len(libs))}
     ref = None
     for r in range(a.rounds + 2):
         for i, h in enumerate(libs):
@@ -78,6 +79,10 @@ def main():
             h.cuszp_range(x.data_ptr(), n, mm.data_ptr(), ws.data_ptr(), ws.numel(), sp)
             h.cuszp_compress_minmax(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, out.data_ptr(), cap, ob.data_ptr(),
                                     ws.data_ptr(), ws.numel(), sp); ev[7].record()
+            # REL as one call (range + compress; the library may overlap them)
+            flush.zero_(); ev[8].record()
+            h.cuszp_compress(x.data_ptr(), n, a.rel, 1, out.data_ptr(), cap, ob.data_ptr(), ws.data_ptr(), ws.numel(),
+                             sp); ev[9].record()
             torch.cuda.synchronize()
             S = int(ob.item())
             digest = (S, float(y[:1000].sum()), float(y[-1000:].sum()))
@@ -88,6 +93,7 @@ def main():
                 res[i]["compress"].append(ev[2].elapsed_time(ev[3]) * 1e3)
                 res[i]["decompress"].append(ev[4].elapsed_time(ev[5]) * 1e3)
                 res[i]["rel_chain"].append(ev[6].elapsed_time(ev[7]) * 1e3)
+                res[i]["rel_call"].append(ev[8].elapsed_time(ev[9]) * 1e3)
     print(f"n={n} S={ref[0]} CR={4 * n / ref[0]:.2f}  (us: median / min)")
     occ = (C.c_int * 4)()
     for p_, h in zip(a.libs, libs):
@@ -98,7 +104,7 @@ def main():
         print(f"{os.path.basename(p):40s} range {np.median(d['range']):7.1f}/{min(d['range']):7.1f}  "
               f"compress {np.median(d['compress']):7.1f}/{min(d['compress']):7.1f}  "
               f"decompress {np.median(d['decompress']):7.1f}/{min(d['decompress']):7.1f}  "
-              f"range+compress {np.median(d['rel_chain']):7.1f}")
+              f"range+compress {np.median(d['rel_chain']):7.1f}  REL call {np.median(d['rel_call']):7.1f}")
 
 
 if __name__ == "__main__":

@@ -64,20 +64,24 @@ static int round_trip(size_t n, float eb, int mode, int L, int order) {
   unsigned long long S = 0;
   CK(cudaMemcpy(&S, d_len, 8, cudaMemcpyDeviceToHost));
   int st = cuszp_last_status(d_ws, nullptr);
+  int bad = 0;
   if (st != CUSZP_OK) {
     std::fprintf(stderr, "n=%zu L=%d order=%d: compress status %s\n", n, L, order, cuszp_status_string(st));
-    return 1;
+    bad = 1;
+    S = 32;
   }
   // decompress from an exact-size copy of the stream (every read must stay inside S bytes)
   CK(cudaMalloc(&d_exact, S));
   CK(cudaMemcpy(d_exact, d_out, S, cudaMemcpyDeviceToDevice));
-  OKS(cuszp_decompress_ex(d_exact, S, d_y, n, L, order, d_ws, wsb, nullptr));
-  st = cuszp_last_status(d_ws, nullptr);
   std::vector<float> y(n);
-  CK(cudaMemcpy(y.data(), d_y, n * sizeof(float), cudaMemcpyDeviceToHost));
   cuszp_header h;
-  CK(cudaMemcpy(&h, d_exact, 32, cudaMemcpyDeviceToHost));
-  int bad = (st != CUSZP_OK);
+  if (!bad) {
+    OKS(cuszp_decompress_ex(d_exact, S, d_y, n, L, order, d_ws, wsb, nullptr));
+    st = cuszp_last_status(d_ws, nullptr);
+    CK(cudaMemcpy(y.data(), d_y, n * sizeof(float), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&h, d_exact, 32, cudaMemcpyDeviceToHost));
+    bad = (st != CUSZP_OK);
+  }
   for (size_t i = 0; i < n && !bad; ++i) {
     const double ulp = double(std::nextafterf(std::fabs(x[i]), INFINITY)) - std::fabs(double(x[i]));
     if (std::fabs(double(x[i]) - double(y[i])) > double(h.eb_abs) + ulp) {
@@ -98,7 +102,7 @@ int main(int argc, char** argv) {
   int fails = 0;
   const size_t sizes[] = {1, 31, 33, 4095, 4097, 100003, (size_t(1) << 20) + 11};
   for (size_t n : sizes) {
-    fails += round_trip(n, 1e-4f, CUSZP_REL, 32, 1);
+    if (n > 1) fails += round_trip(n, 1e-4f, CUSZP_REL, 32, 1);     // n = 1 is a constant field: ERANGE by R5
     fails += round_trip(n, 1e-3f, CUSZP_ABS, 32, 1);
   }
   fails += round_trip(100003, 1e-4f, CUSZP_REL, 64, 1);

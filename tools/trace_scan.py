@@ -130,6 +130,21 @@ def main():
     pk = trace[nt * 16:].view(nt, 8).cpu().numpy().astype(np.int64)
     busy = (pw - pk) / 1e3
     print("decompress per-warp tile compute (pickup -> done, us):", pct(busy.ravel()))
+    # per CTA (slot 7) and warp: idle gap between finishing one tile and picking up the next
+    cta = trd[:, 7]
+    gaps, waits = [], []
+    for c in np.unique(cta):
+        idx = np.nonzero(cta == c)[0]
+        idx = idx[np.argsort(pk[idx, 0])]
+        for wv in range(8):
+            g = (pk[idx[1:], wv] - pw[idx[:-1], wv]) / 1e3
+            gaps.append(g)
+            waits.append((pk[idx[1:], wv] - np.maximum(pw[idx[:-1], wv], trd[idx[1:], 3])) / 1e3)
+    gaps = np.concatenate(gaps)
+    print("decompress per-warp gap done(k) -> pickup(k+1) (us):", pct(gaps), f" mean {gaps.mean():.2f}")
+    print("   of which after the next tile's TMA was issued (us):", pct(np.concatenate(waits)))
+    span = (pw.max() - pk.min()) / 1e3
+    print(f"   warp busy fraction: {busy.sum() / (span * 8 * len(np.unique(cta))):.2f}")
     # per warp slot, consecutive tiles of the same CTA are not identifiable; use the
     # distribution of each warp's pickup relative to the tile's TMA issue instead
     wait = (pk - trd_issue[:, None]) / 1e3 if False else None
