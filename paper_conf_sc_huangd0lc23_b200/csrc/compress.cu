@@ -54,6 +54,10 @@ namespace {
 #ifndef CUSZP_C_MINBLOCKS
 #define CUSZP_C_MINBLOCKS (CUSZP_C_CW > 8 ? 2 : 3)
 #endif
+#ifndef CUSZP_C_GUNROLL
+#define CUSZP_C_GUNROLL 4
+#endif
+constexpr int kGUnroll = CUSZP_C_GUNROLL;         // groups of 4 blocks unrolled in the encode loop
 constexpr int kStages = CUSZP_C_STAGES;          // input ring depth (16 KB tiles)
 constexpr int kWriters = CUSZP_C_WRITERS;        // scan + writer warps
 constexpr int kMeta = CUSZP_C_META;              // tiles between "computed" and "released"
@@ -542,7 +546,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         // else 1.  After it, lane q*W + k holds word k of block q (W = 32 /
         // blocks per transpose), and a ballot of the non-zero words gives every
         // block's word count (the top plane is non-zero by definition of F).
-#pragma unroll
+#pragma unroll kGUnroll
 #ifdef CUSZP_DIAG_NOWORK
         for (int g = 0; g < 0; ++g) {   // diagnostics only: pipeline without the encode work
 #else
@@ -679,15 +683,21 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             }
           }
           cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
+#if CUSZP_C_GUNROLL >= 4
           wbs[g] = wb;
+#else
+          if (lane == 0) sm.meta[m].wb[w * (kCBPW / 4) + g] = wb;  // sync: acq_rel count, then mbarrier staged[m]
+#endif
         }
         __syncwarp();
         if (lane == 0) {
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
           TileMeta& md = sm.meta[m];
           // the group word counts go to the writer, which stores the tile's F bytes
+#if CUSZP_C_GUNROLL >= 4
           if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           else *reinterpret_cast<uint2*>(&md.wb[w * 2]) = make_uint2(wbs[0], wbs[1]);  // sync: acq_rel count, then mbarrier staged[m]
+#endif
           md.cnt[w] = uint16_t(cursor);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           md.head[w] = uint16_t(head & (kRing - 1));  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           uint32_t done;                                   // release: cnt/head before the count; acquire: the others'
