@@ -71,18 +71,22 @@ static_assert(kCW == 8 || kCW == 16, "compute warps");
 constexpr int kCThreads = (kFirstCompute + kCW) * 32;
 static_assert((kRing & (kRing - 1)) == 0 && kRing >= 4 * 32, "ring size");
 
+// WB = words of packed per-block plane counts per tile: 32 for L >= 32 (the
+// 128 sub-blocks), 128 / 64 for L = 8 / 16 (512 / 256 blocks)
+template <int WB>
 struct alignas(16) TileMeta {
-  uint32_t wb[kTileBlocks / 4];    // words of the 4 sub-blocks of every group (bytes), tile order
+  uint32_t wb[WB];                 // plane counts (= F + 1, 0 for a zero block) of 4 blocks (bytes), tile order
   uint32_t tile;
-  uint32_t agg;                    // words of the tile
-  uint16_t cnt[kCW];               // words per compute warp
-  uint16_t head[kCW];              // ring position of each warp's first word
+  uint32_t agg;                    // words of the tile (bytes for L = 8 / 16)
+  uint16_t cnt[kCW];               // words (bytes) per compute warp
+  uint16_t head[kCW];              // ring position of each warp's first word (byte)
 };
 
+template <int WB>
 struct CompressSmem {
-  float in[kStages][kTileElems];                 // 48 KB
+  float in[kStages][kTileElems];                 // 32 KB
   uint32_t ring[kCW][kRing];                     // 4 KB per compute warp
-  TileMeta meta[kMeta];
+  TileMeta<WB> meta[kMeta];
   uint32_t in_tile[kStages];
   uint32_t meta_done[kMeta];
   uint32_t tail[kCW];                            // ring words released (monotonic)
@@ -243,18 +247,98 @@ __device__ __forceinline__ uint32_t lorenzo_md_pack(uint32_t rb, int lane) {
   return (a << 1) | (uint32_t(l) >> 31);
 }
 
+// L = 8 / 16 (SL): a 32-lane row holds BR = 32 / SL blocks and a plane of a
+// block is SL / 8 BYTES (element j at byte j / 8, bit j % 8, R9
+// generalised), so a transposed word holds one plane of BR blocks: byte
+// (L = 8) or halfword (L = 16) b is block b's.  One group = 4 rows = 4 BR
+// blocks.  S rows share a transpose (S = 4 when every v < 2^8, 2 when
+// < 2^16, else 1): lane 32/S * h + k then holds plane k of row S p + h.
+//   plane counts: a ballot of "part b non-zero" over the planes of a row
+//                 segment, bit length (= F + 1, 0 for a zero block, Eq 2);
+//   offsets:      segmented scan of the block byte counts over the group;
+//   sequences:    a 4 x 4 byte (L = 8) / 2 x 2 halfword (L = 16) transpose
+//                 inside lane quads / pairs turns lane BR m + b of a segment
+//                 into bytes 4m .. 4m+3 of block b's byte sequence (sign map
+//                 then planes), stored bytewise at the block's
+//                 offset in the warp's byte ring.
+// Writes the group's packed plane counts to wb[0 .. BR-1]; returns its bytes.
+template <int SL, int S>
+__device__ __forceinline__ uint32_t place_small(const uint32_t (&v)[4], const Xpose& xpose, int lane,
+                                                uint8_t* ringb, uint32_t base, uint32_t* wb) {
+  constexpr int BR = 32 / SL, NBG = 4 * BR, NX = 4 / S, SEG = 32 / S, PB = SL / 8;
+  constexpr uint32_t kMaskB = kRing * 4 - 1;
+  uint32_t tw[NX];
+#pragma unroll
+  for (int p = 0; p < NX; ++p) {
+    const uint32_t x = (S == 4) ? pack4(v[0], v[1], v[2], v[3])
+                     : (S == 2) ? __byte_perm(v[2 * p], v[2 * p + 1], 0x5410u) : v[p];
+    tw[p] = xpose(x);
+  }
+  // plane count of block beta = lane % NBG (row beta / BR, part beta % BR)
+  const int beta = lane % NBG, row = beta / BR, part = beta % BR;
+  uint32_t bal = 0;
+#pragma unroll
+  for (int p = 0; p < NX; ++p)
+#pragma unroll
+    for (int b = 0; b < BR; ++b) {
+      const uint32_t pm = (SL == 8 ? 0xffu : 0xffffu) << (8 * PB * b);
+      const uint32_t bb = __ballot_sync(kFull, (tw[p] & pm) != 0u);
+      if (p == row / S && b == part) bal = bb;
+    }
+  const uint32_t segbits = (SEG == 32) ? bal : (bal >> (SEG * (row % S))) & ((1u << (SEG & 31)) - 1u);
+  const uint32_t planes = 32u - __clz(segbits);
+  const uint32_t bytes = planes * PB;
+  uint32_t incl = bytes;
+#pragma unroll
+  for (int o = 1; o < NBG; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(kFull, incl, o, NBG);
+    if (beta >= o) incl += y;
+  }
+  const uint32_t info = (incl - bytes) | (bytes << 16);          // exclusive offset | bytes
+  const uint32_t gbytes = __shfl_sync(kFull, incl, NBG - 1);
+  uint32_t f = planes << (8 * (beta & 3));                       // 4 blocks' plane counts per word
+  f |= __shfl_xor_sync(kFull, f, 1);
+  f |= __shfl_xor_sync(kFull, f, 2);
+  if (lane < NBG && (lane & 3) == 0) wb[lane >> 2] = f;  // sync: acq_rel count, then mbarrier staged[m]
+  const int k = lane % SEG;
+  const uint32_t m = uint32_t(k / BR), b = uint32_t(k % BR);
+#pragma unroll
+  for (int p = 0; p < NX; ++p) {
+    uint32_t x = tw[p];
+    if constexpr (SL == 8) {                                     // 4 x 4 byte transpose in lane quads
+      x = __byte_perm(x, __shfl_xor_sync(kFull, x, 2), (lane & 2) ? 0x3276u : 0x5410u);
+      x = __byte_perm(x, __shfl_xor_sync(kFull, x, 1), (lane & 1) ? 0x3715u : 0x6240u);
+    } else {                                                     // 2 x 2 halfword transpose in lane pairs
+      x = __byte_perm(x, __shfl_xor_sync(kFull, x, 1), (lane & 1) ? 0x3276u : 0x5410u);
+    }
+    const uint32_t src = uint32_t(S * p + lane / SEG) * BR + b;  // block of this lane's chunk
+    const uint32_t in = __shfl_sync(kFull, info, int(src));
+    const uint32_t nb = in >> 16, pos = base + (in & 0xffffu) + 4 * m;
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      if (4 * m + j < nb) ringb[(pos + j) & kMaskB] = uint8_t(x >> (8 * j));  // sync: ring slot freed by the writer's tail release; read after staged[m]
+  }
+  return gbytes;
+}
+
 // O = Lorenzo order: 1 (the paper's 1D 1-layer predictor) or 2 (2-layer,
 // SURVEY 8(f) rank 4; L = 32 only).
 // D = Lorenzo dimensions (DESIGN R18): 1 = the paper's 1D
 // predictor over consecutive elements; 2 / 3 = blocks of 1x4x8 / 2x4x4 points
 // of an (nz, ny, nx) field, gathered into tile order by the producer warp.
-template <int M, int O, int D = 1>
+// SL = 8 / 16: the byte-granular block lengths (place_small; M = 1): the
+// look-back, rings and copy-out count BYTES instead of words.
+template <int M, int O, int D = 1, int SL = 0>
 __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(CompressArgs a) {
   static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
   static_assert(D == 1 || (M == 1 && O == 1), "multi-dimensional Lorenzo with L = 32, order 1");
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
+  static_assert(SL == 0 || ((SL == 8 || SL == 16) && M == 1 && O == 1 && D == 1), "L = 8 / 16");
+  constexpr bool kSmall = SL != 0;
+  constexpr int kWB = kSmall ? kTileElems / SL / 4 : kTileBlocks / 4;
+  constexpr uint32_t kSegMask = (kSmall ? SL : 32) - 1;   // lane bits inside a block (Lorenzo restarts)
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  CompressSmem& sm = *reinterpret_cast<CompressSmem*>(smem_raw);
+  CompressSmem<kWB>& sm = *reinterpret_cast<CompressSmem<kWB>*>(smem_raw);
   const int lane = threadIdx.x & 31;
   const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);   // provably warp-uniform (no divergence checks before warp-sync ops)
   pdl_wait();                                     // range kernel / previous call complete
@@ -433,16 +517,30 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #endif
         const uint64_t excl = resolve_excl(a.status, t, epoch, &nw, &ns);
         mbar_wait(&sm.staged[m], par);                      // suspending wait: no issue slots taken
-        const TileMeta& md = sm.meta[m];
+        const TileMeta<kWB>& md = sm.meta[m];
         const uint32_t agg = md.agg;  // sync: mbarrier staged[m]
         if (lane == 0 && t > 0) publish_prefix(a.status, t, excl + agg, epoch);
-        {
+        auto fbytes = [](uint32_t wb) { return wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u); };
+        if constexpr (kSmall) {
+          // F bytes: 512 / 256 per tile, 16 / 8 per lane (plane counts -> F bytewise)
+          constexpr uint32_t kPer = uint32_t(kWB) / 32u;
+          const uint64_t blk = uint64_t(t) * (kTileElems / SL) + 4u * kPer * lane;
+          if (blk < align16(a.nb)) {
+            if constexpr (kPer == 4) {
+              const uint4 q = *reinterpret_cast<const uint4*>(&md.wb[4 * lane]);  // sync: mbarrier staged[m] after the compute warps' acq_rel count
+              *reinterpret_cast<uint4*>(a.out + kHdr + blk) = make_uint4(fbytes(q.x), fbytes(q.y), fbytes(q.z), fbytes(q.w));
+            } else {
+              const uint2 q = *reinterpret_cast<const uint2*>(&md.wb[2 * lane]);  // sync: mbarrier staged[m] after the compute warps' acq_rel count
+              *reinterpret_cast<uint2*>(a.out + kHdr + blk) = make_uint2(fbytes(q.x), fbytes(q.y));
+            }
+          }
+        } else {
           // F bytes of the tile (Fig 12 part 1): lane L converts group L's word
           // counts, F = words - 1 (0 for a zero block) bytewise (counts <= 32, no
           // carries); the stores also cover the F area's zero padding up to
           // align16(nb) (sub-blocks past n encode as zero blocks, F = 0)
           const uint32_t wb = md.wb[lane];  // sync: mbarrier staged[m] after the compute warps' acq_rel count
-          uint32_t f = wb - (((wb + 0x7f7f7f7fu) >> 7) & 0x01010101u);
+          const uint32_t f = fbytes(wb);
           const uint64_t blk = (uint64_t(t) * kTileBlocks + 4u * lane) / M;
           if (blk < align16(a.nb)) {
             if constexpr (M == 1) *reinterpret_cast<uint32_t*>(a.out + kHdr + blk) = f;
@@ -469,6 +567,36 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         // a8 store: each compute warp's ring segment -> [excl + warp offset, ...):
         // the segment is at most two linear pieces of the ring (before and
         // after its wrap point), each copied with running pointers
+        if constexpr (kSmall) {
+          // byte segments: the (<= 3) bytes before the first 4-byte aligned
+          // destination word and after the last go bytewise (they share words
+          // with the neighbouring segments / tiles); the words in between are
+          // funnel-shifted out of two ring words
+          constexpr uint32_t kMaskB = kRing * 4 - 1;
+          const uint8_t* ringb_all = reinterpret_cast<const uint8_t*>(sm.ring);
+#pragma unroll 1
+          for (int w = 0; w < kCW; ++w) {
+            const uint32_t c = __shfl_sync(kFull, cnt, w);
+            const uint32_t h = __shfl_sync(kFull, hd, w);
+            const uint32_t off = __shfl_sync(kFull, incl - cnt, w);
+            const uint8_t* rb = ringb_all + w * (kRing * 4);
+            const uint32_t* rw = sm.ring[w];
+            uint8_t* g = a.out + p0 + excl + off;
+            const uint32_t hb = min(c, uint32_t(-reinterpret_cast<uintptr_t>(g)) & 3u);
+            const uint32_t nw = (c - hb) >> 2, tb = c - hb - 4 * nw;
+            if (uint32_t(lane) < hb) g[lane] = rb[(h + lane) & kMaskB];  // sync: ring written before staged[m]; reused only after the tail release
+            if (uint32_t(lane) < tb) g[hb + 4 * nw + lane] = rb[(h + hb + 4 * nw + lane) & kMaskB];  // sync: ring written before staged[m]; reused only after the tail release
+            const uint32_t s0 = h + hb, sh = 8 * (s0 & 3u);
+            uint32_t* gw = reinterpret_cast<uint32_t*>(g + hb);
+#pragma unroll 2
+            for (uint32_t k = lane; k < nw; k += 32) {
+              const uint32_t wi = (s0 >> 2) + k;
+              const uint32_t lo = rw[wi & (kRing - 1)];  // sync: ring written before staged[m]; reused only after the tail release
+              const uint32_t hi = rw[(wi + 1) & (kRing - 1)];  // sync: ring written before staged[m] (bytes past the segment unused)
+              gw[k] = __funnelshift_r(lo, hi, sh);
+            }
+          }
+        } else {
         uint32_t* dst_t = payload + excl + lane;
 #pragma unroll 1
         for (int w = 0; w < kCW; ++w) {
@@ -484,6 +612,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           dst = dst_t + off + first;
 #pragma unroll 2
           for (int k = lane; k < int(c - first); k += 32, src += 32, dst += 32) *dst = *src;  // sync: ring written before staged[m]; reused only after the tail release
+        }
         }
         // release ring space in CTA tile order
         if (lane == 0) stress_delay(j ^ 0x55u);
@@ -503,7 +632,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       const Xpose xpose(lane);
       // scaled-float Lorenzo (quantize_scaled2) for the paper's default L = 32, order 1
       constexpr bool kScaled = (M == 1 && O == 1 && D == 1);
-      const float kf = lane ? -1.0f : -0.0f;
+      const float kf = (uint32_t(lane) & kSegMask) ? -1.0f : -0.0f;   // -0: the lane starts a block
       const uint64_t nk = (uint64_t(__float_as_uint(kf)) << 32) | __float_as_uint(kf);
       uint32_t head = 0;                                // words this warp has appended (monotonic)
       uint32_t* ring = sm.ring[w];
@@ -539,7 +668,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         uint32_t cursor = 0;
         // free words in this warp's ring (refreshed only when a worst-case
         // group would not fit)
-        uint32_t room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
+        uint32_t room = (kSmall ? kRing * 4 : kRing) - (head - ld_volatile_u32(&sm.tail[w]));
         uint32_t wbs[kCBPW / 4];                       // word counts of each group (bytes), for the F array
         // Groups of 4 blocks.  The bit transpose packs as many blocks as fit
         // in 32 bits: 4 blocks when every v < 2^8 (F <= 7), 2 when v < 2^16,
@@ -584,14 +713,18 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           uint32_t v[4], wq[4];
           auto counts = [&]() {
             // a5: words per block = bit length of the block's OR of v (= of its max)
+            // (L = 8 / 16: counted after the transpose, place_small)
+            if constexpr (!kSmall) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) wq[q] = 32u - __clz(__reduce_or_sync(kFull, v[q]));
+              for (int q = 0; q < 4; ++q) wq[q] = 32u - __clz(__reduce_or_sync(kFull, v[q]));
+            }
           };
           auto lorenzo_and_counts = [&]() {
             if constexpr (M == 1) {
 #pragma unroll
               for (int q = 0; q < 4; ++q)
-                v[q] = (D > 1) ? lorenzo_md_pack<D>(r[q], lane) : (O == 2) ? lorenzo2_pack(r[q], lane) : lorenzo_pack(r[q], lane);
+                v[q] = (D > 1) ? lorenzo_md_pack<D>(r[q], lane) : (O == 2) ? lorenzo2_pack(r[q], lane)
+                                                                   : lorenzo_pack(r[q], int(uint32_t(lane) & kSegMask));
             } else {
               // a block continues across its sub-blocks: lane 0 of sub-block q
               // takes lane 31 of sub-block q-1 unless q starts a block
@@ -619,87 +752,104 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             lorenzo_and_counts();
           }
 #endif
-          // room in this warp's ring for a worst-case group (4 x 32 words)
-          while (cursor + 4 * 32 > room) {
-            room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
-            if (cursor + 4 * 32 > room) __nanosleep(CUSZP_C_POLL_NS);
-          }
-          if constexpr (M == 2) {                                        // one F per block
-            wq[0] = wq[1] = max(wq[0], wq[1]);
-            wq[2] = wq[3] = max(wq[2], wq[3]);
-          } else if constexpr (M == 4) {
-            wq[0] = wq[1] = wq[2] = wq[3] = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
-          }
-          // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
-          // flagged ERANGE at the end.  Such garbage blocks still take at most
-          // 32 words (v is 32-bit), which the capacity bound covers (DESIGN 9.5).
-          const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
-          wmax = max(wmax, span);
-          const uint32_t wb = pack4(wq[0], wq[1], wq[2], wq[3]);
-          const uint32_t base = head + cursor;
-          if (M > 1) {
-            // word k of sub-block q -> block payload position M k + q % M
-            const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
-            if (span <= 8) {
+          if constexpr (kSmall) {
+            const uint32_t span = 32u - __clz(__reduce_or_sync(kFull, v[0] | v[1] | v[2] | v[3]));
+            wmax = max(wmax, span);
+            // room for a worst-case group (4 BR blocks x 32 planes x SL/8 bytes = 512 bytes)
+            while (cursor + 512 > room) {
+              room = kRing * 4 - (head - ld_volatile_u32(&sm.tail[w]));
+              if (cursor + 512 > room) __nanosleep(CUSZP_C_POLL_NS);
+            }
+            uint8_t* ringb = reinterpret_cast<uint8_t*>(ring);
+            uint32_t* wbg = &sm.meta[m].wb[(w * (kCBPW / 4) + g) * (32 / SL)];
+            const uint32_t base = head + cursor;
+            if (span <= 8) cursor += place_small<SL, 4>(v, xpose, lane, ringb, base, wbg);
+            else if (span <= 16) cursor += place_small<SL, 2>(v, xpose, lane, ringb, base, wbg);
+            else cursor += place_small<SL, 1>(v, xpose, lane, ringb, base, wbg);
+          } else {
+            // room in this warp's ring for a worst-case group (4 x 32 words)
+            while (cursor + 4 * 32 > room) {
+              room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
+              if (cursor + 4 * 32 > room) __nanosleep(CUSZP_C_POLL_NS);
+            }
+            if constexpr (M == 2) {                                        // one F per block
+              wq[0] = wq[1] = max(wq[0], wq[1]);
+              wq[2] = wq[3] = max(wq[2], wq[3]);
+            } else if constexpr (M == 4) {
+              wq[0] = wq[1] = wq[2] = wq[3] = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+            }
+            // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
+            // flagged ERANGE at the end.  Such garbage blocks still take at most
+            // 32 words (v is 32-bit), which the capacity bound covers (DESIGN 9.5).
+            const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+            wmax = max(wmax, span);
+            const uint32_t wb = pack4(wq[0], wq[1], wq[2], wq[3]);
+            const uint32_t base = head + cursor;
+            if (M > 1) {
+              // word k of sub-block q -> block payload position M k + q % M
+              const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
+              if (span <= 8) {
+                const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
+                const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
+                const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
+                if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              } else if (span <= 16) {
+                const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
+                const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
+                const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
+                if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+                const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
+                const uint32_t sub23 = (M == 2) ? h : 2u + h;
+                if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                  const uint32_t tq = xpose(v[q]);
+                  const uint32_t pre = (q & ~(M - 1)) == 0 ? 0u : __byte_perm(pb, 0, 0x4440u + (q & ~(M - 1)));
+                  if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+                }
+              }
+            } else if (span <= 8) {
               const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
-              const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
-              const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
-              if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
+              const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
+              if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             } else if (span <= 16) {
               const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
               const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
-              const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
-              if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-              const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
-              const uint32_t sub23 = (M == 2) ? h : 2u + h;
-              if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              const bool hi = lane >= 16;
+              const uint32_t k = lane & 15;
+              if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             } else {
+              uint32_t o = base;
 #pragma unroll
               for (int q = 0; q < 4; ++q) {
                 const uint32_t tq = xpose(v[q]);
-                const uint32_t pre = (q & ~(M - 1)) == 0 ? 0u : __byte_perm(pb, 0, 0x4440u + (q & ~(M - 1)));
-                if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+                if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+                o += wq[q];
               }
             }
-          } else if (span <= 8) {
-            const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
-            const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
-            const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
-            if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-          } else if (span <= 16) {
-            const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
-            const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
-            const bool hi = lane >= 16;
-            const uint32_t k = lane & 15;
-            if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-            if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-          } else {
-            uint32_t o = base;
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              const uint32_t tq = xpose(v[q]);
-              if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-              o += wq[q];
-            }
-          }
-          cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
+            cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
 #if CUSZP_C_GUNROLL >= 4
-          wbs[g] = wb;
+            wbs[g] = wb;
 #else
-          if (lane == 0) sm.meta[m].wb[w * (kCBPW / 4) + g] = wb;  // sync: acq_rel count, then mbarrier staged[m]
+            if (lane == 0) sm.meta[m].wb[w * (kCBPW / 4) + g] = wb;  // sync: acq_rel count, then mbarrier staged[m]
 #endif
+          }
         }
         __syncwarp();
         if (lane == 0) {
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
-          TileMeta& md = sm.meta[m];
+          TileMeta<kWB>& md = sm.meta[m];
           // the group word counts go to the writer, which stores the tile's F bytes
 #if CUSZP_C_GUNROLL >= 4
-          if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
+          if constexpr (kSmall) {}
+          else if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           else *reinterpret_cast<uint2*>(&md.wb[w * 2]) = make_uint2(wbs[0], wbs[1]);  // sync: acq_rel count, then mbarrier staged[m]
 #endif
           md.cnt[w] = uint16_t(cursor);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
-          md.head[w] = uint16_t(head & (kRing - 1));  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
+          md.head[w] = uint16_t(head & ((kSmall ? 4 * kRing : kRing) - 1));  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           uint32_t done;                                   // release: cnt/head before the count; acquire: the others'
           asm volatile("atom.acq_rel.cta.shared::cta.add.u32 %0, [%1], 1;"
                        : "=r"(done) : "r"(smem_u32(&sm.meta_done[m])) : "memory");
@@ -737,13 +887,13 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       uint64_t total_words = 0;
       if (final_status == CUSZP_OK && a.num_tiles > 0)
         total_words = ld_relaxed_u64(a.status + a.num_tiles - 1) & kValueMask;
-      const uint64_t payload_bytes = final_status == CUSZP_OK ? total_words * 4 : 0;
+      const uint64_t payload_bytes = final_status == CUSZP_OK ? total_words * (kSmall ? 1 : 4) : 0;   // L = 8 / 16 count bytes
       uint8_t* h = a.out;                                   // header (R10)
       *reinterpret_cast<uint32_t*>(h) = 0x505A5343u;        // "CSZP"
       h[4] = CUSZP_VERSION;
       h[5] = uint8_t(a.mode | (O == 2 ? 0x10 : 0) | ((D - 1) << 5));   // predictor order (R17), dims (R18)
       h[6] = uint8_t(final_status);
-      h[7] = uint8_t(5 + (M == 2 ? 1 : M == 4 ? 2 : 0));   // log2(L)
+      h[7] = uint8_t(SL == 8 ? 3 : SL == 16 ? 4 : 5 + (M == 2 ? 1 : M == 4 ? 2 : 0));   // log2(L)
       *reinterpret_cast<uint64_t*>(h + 8) = a.n;
       // R11: n = 0 records the bound that would have been used (a sharded
       // REL shard's global lambda * range; 0 for a lone empty REL array)
@@ -757,43 +907,60 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 }
 
 namespace {
-template <int M, int O = 1, int D = 1>
+template <int M, int O = 1, int D = 1, int SL = 0>
 cudaError_t configure_m(int* occ) {
-  const int smem = int(sizeof(CompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M, O, D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M, O, D>, kCThreads, smem);
+  constexpr int kWB = SL ? kTileElems / SL / 4 : kTileBlocks / 4;
+  const int smem = int(sizeof(CompressSmem<kWB>));
+  cudaError_t e = cudaFuncSetAttribute(compress_kernel<M, O, D, SL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, compress_kernel<M, O, D, SL>, kCThreads, smem);
   return e;
+}
+template <int M, int O = 1, int D = 1, int SL = 0>
+cudaError_t launch_k(cudaLaunchConfig_t cfg, const CompressArgs& a) {
+  constexpr int kWB = SL ? kTileElems / SL / 4 : kTileBlocks / 4;
+  cfg.dynamicSmemBytes = sizeof(CompressSmem<kWB>);
+  return cudaLaunchKernelEx(&cfg, compress_kernel<M, O, D, SL>, a);
 }
 }  // namespace
 
-cudaError_t compress_configure(int M, int* occ) {
+// L in {8, 16, 32, 64, 128}: resident CTAs per SM of that block length's kernel
+cudaError_t compress_configure(int L, int* occ) {
   int occ2 = 0;
-  if (M == 1 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
-                 configure_m<1, 1, 3>(&occ2) != cudaSuccess))
+  if (L == 32 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
+                  configure_m<1, 1, 3>(&occ2) != cudaSuccess))
     return cudaErrorUnknown;
-  return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
+  switch (L) {
+    case 8: return configure_m<1, 1, 1, 8>(occ);
+    case 16: return configure_m<1, 1, 1, 16>(occ);
+    case 32: return configure_m<1>(occ);
+    case 64: return configure_m<2>(occ);
+    default: return configure_m<4>(occ);
+  }
 }
 
-cudaError_t compress_launch(int M, int order, unsigned grid, const CompressArgs& a, cudaStream_t s) {
+cudaError_t compress_launch(int L, int order, unsigned grid, const CompressArgs& a, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kCThreads);
-  cfg.dynamicSmemBytes = sizeof(CompressSmem);
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;   // see pdl_wait()
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (a.dims == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1, 2>, a);
-  if (a.dims == 3) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1, 3>, a);
-  if (order == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 2>, a);
-  if (M == 1) return cudaLaunchKernelEx(&cfg, compress_kernel<1, 1>, a);
-  if (M == 2) return cudaLaunchKernelEx(&cfg, compress_kernel<2, 1>, a);
-  return cudaLaunchKernelEx(&cfg, compress_kernel<4, 1>, a);
+  if (a.dims == 2) return launch_k<1, 1, 2>(cfg, a);
+  if (a.dims == 3) return launch_k<1, 1, 3>(cfg, a);
+  if (order == 2) return launch_k<1, 2>(cfg, a);
+  switch (L) {
+    case 8: return launch_k<1, 1, 1, 8>(cfg, a);
+    case 16: return launch_k<1, 1, 1, 16>(cfg, a);
+    case 32: return launch_k<1, 1>(cfg, a);
+    case 64: return launch_k<2, 1>(cfg, a);
+    default: return launch_k<4, 1>(cfg, a);
+  }
 }
 
-size_t compress_smem_bytes() { return sizeof(CompressSmem); }
+size_t compress_smem_bytes() { return sizeof(CompressSmem<kTileBlocks / 4>); }
 int compress_threads() { return kCThreads; }
 
 }  // namespace cuszp

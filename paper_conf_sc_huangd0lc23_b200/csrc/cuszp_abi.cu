@@ -23,7 +23,8 @@ uint64_t num_tiles(uint64_t n) { return (num_blocks(n) + kTileBlocks - 1) / kTil
 struct DeviceInfo {
   int sms = 0;
   int occ_compress = 0, occ_decompress = 0, occ_range = 0, occ_quality = 0;
-  int occ_c[3] = {0, 0, 0}, occ_d[3] = {0, 0, 0};   // per M = 1, 2, 4
+  int occ_c[5] = {0, 0, 0, 0, 0};   // compress, per L = 8, 16, 32, 64, 128
+  int occ_d[3] = {0, 0, 0};         // decompress, per M = 1, 2, 4
 };
 
 // Per-device launch geometry, computed once: persistent grids of
@@ -38,15 +39,14 @@ int device_info(DeviceInfo* out) {
   if (!have[dev]) {
     DeviceInfo d;
     if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return CUSZP_ECUDA;
-    for (int k = 0; k < 3; ++k) {
-      const int M = 1 << k;
-      if (compress_configure(M, &d.occ_c[k]) != cudaSuccess || decompress_configure(M, &d.occ_d[k]) != cudaSuccess)
-        return CUSZP_ECUDA;
-    }
+    for (int k = 0; k < 5; ++k)
+      if (compress_configure(8 << k, &d.occ_c[k]) != cudaSuccess) return CUSZP_ECUDA;
+    for (int k = 0; k < 3; ++k)
+      if (decompress_configure(1 << k, &d.occ_d[k]) != cudaSuccess) return CUSZP_ECUDA;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_quality, quality_kernel, 256, 0) != cudaSuccess)
       return CUSZP_ECUDA;
-    d.occ_compress = d.occ_c[0];
+    d.occ_compress = d.occ_c[2];
     d.occ_decompress = d.occ_d[0];
     cache[dev] = d;
     have[dev] = true;
@@ -133,13 +133,16 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   a.status = reinterpret_cast<uint64_t*>(static_cast<uint8_t*>(d_ws) + kWsCtrlBytes);
   a.status_cap = status_capacity(ws_bytes);
   a.trace = g_trace;
+#ifdef CUSZP_SMALL_L_3PASS
+  // diagnostics build: the three-launch L = 8 / 16 path (small_l.cu), for A/B
   if (small_L(L)) return compress_small_launch(L, a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
-  const int occ = di.occ_c[mi(M)];
+#endif
+  const int occ = di.occ_c[L == 8 ? 0 : L == 16 ? 1 : 2 + mi(M)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_compress > 0) grid = uint64_t(g_grid_compress);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  return compress_launch(M, order, unsigned(grid), a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+  return compress_launch(L, order, unsigned(grid), a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
 }  // namespace

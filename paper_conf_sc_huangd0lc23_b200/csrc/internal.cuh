@@ -468,8 +468,8 @@ constexpr int kQualityMaxGrid = 2048;
 
 // Kernels templated on M = L / 32 are launched through these host wrappers
 // defined next to them (compress.cu / decompress.cu): M in {1, 2, 4}.
-cudaError_t compress_configure(int M, int* occupancy);        // smem attribute + CTAs per SM
-cudaError_t compress_launch(int M, int order, unsigned grid, const CompressArgs& a, cudaStream_t s);
+cudaError_t compress_configure(int L, int* occupancy);        // smem attribute + CTAs per SM (L = block length)
+cudaError_t compress_launch(int L, int order, unsigned grid, const CompressArgs& a, cudaStream_t s);
 cudaError_t decompress_configure(int M, int* occupancy);
 cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s);
 // L in {8, 16} (small_l.cu): three launches each, one thread per L-block.

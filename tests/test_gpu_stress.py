@@ -101,6 +101,8 @@ def test_grid_size_sweep_matches_oracle():
             for name, x_np in xs.items():
                 _check(h, x_np, 1e-3, label=f"grid={g} {name}")
             _check(h, xs["walk"], 1e-4, L=64, label=f"grid={g} L=64")
+            _check(h, xs["walk"], 1e-4, L=8, label=f"grid={g} L=8")
+            _check(h, xs["hurricane_U"], 1e-3, L=16, label=f"grid={g} L=16")
             _check(h, xs["walk"], 1e-4, order=2, label=f"grid={g} order=2")
     finally:
         h.cuszp_debug_set_grid(0, 0)
@@ -127,6 +129,8 @@ def test_stress_build_matches_oracle(stress_lib):
                 for name, x_np in xs.items():
                     _check(h, x_np, 1e-3, label=f"stress grid={g} rep={rep} {name}")
             _check(h, xs["hurricane_U"], 1e-4, L=128, label=f"stress grid={g} L=128")
+            _check(h, xs["walk"], 1e-3, L=8, label=f"stress grid={g} L=8")
+            _check(h, xs["qcloud"], 1e-4, L=16, label=f"stress grid={g} L=16")
             _check(h, xs["hurricane_U"], 1e-3, order=2, label=f"stress grid={g} order=2")
     finally:
         h.cuszp_debug_set_grid(0, 0)

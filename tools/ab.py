@@ -22,6 +22,10 @@ def load(path):
     h.cuszp_decompress.argtypes = [vp, sz, vp, sz, vp, sz, vp]
     h.cuszp_workspace_bytes.argtypes = [sz]; h.cuszp_workspace_bytes.restype = sz
     h.cuszp_max_compressed_bytes.argtypes = [sz]; h.cuszp_max_compressed_bytes.restype = sz
+    h.cuszp_max_compressed_bytes_L.argtypes = [sz, i32]; h.cuszp_max_compressed_bytes_L.restype = sz
+    h.cuszp_compress_minmax_L.argtypes = [vp, sz, f32, vp, i32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_compress_L.argtypes = [vp, sz, f32, i32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_decompress_L.argtypes = [vp, sz, vp, sz, i32, vp, sz, vp]
     return h
 
 
@@ -33,6 +37,7 @@ def main():
     ap.add_argument("--field", default=None)
     ap.add_argument("--rel", type=float, default=1e-2)
     ap.add_argument("--nocheck", action="store_true")
+    ap.add_argument("--L", type=int, default=32, help="block length (8, 16, 32, 64, 128)")
     ap.add_argument("--dirty-flush", action="store_true")
     a = ap.parse_args()
     import synth
@@ -42,7 +47,8 @@ def main():
     libs = [load(p) for p in a.libs]
     h0 = libs[0]
     ws = torch.zeros(max(l.cuszp_workspace_bytes(n) for l in libs), dtype=torch.uint8, device=dev)
-    cap = max(l.cuszp_max_compressed_bytes(n) for l in libs)
+    cap = max(l.cuszp_max_compressed_bytes_L(n, a.L) for l in libs)
+    L = a.L
     out = torch.empty(cap, dtype=torch.uint8, device=dev)
     ob = torch.zeros(1, dtype=torch.int64, device=dev)
     mm = torch.empty(2, dtype=torch.float32, device=dev)
@@ -70,19 +76,19 @@ def main():
             flush.zero_(); ev[0].record()
             h.cuszp_range(x.data_ptr(), n, mm.data_ptr(), ws.data_ptr(), ws.numel(), sp); ev[1].record()
             flush.zero_(); ev[2].record()
-            h.cuszp_compress_minmax(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, out.data_ptr(), cap, ob.data_ptr(),
-                                    ws.data_ptr(), ws.numel(), sp); ev[3].record()
+            h.cuszp_compress_minmax_L(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, L, out.data_ptr(), cap, ob.data_ptr(),
+                                      ws.data_ptr(), ws.numel(), sp); ev[3].record()
             flush.zero_(); ev[4].record()
-            h.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.data_ptr(), ws.numel(), sp); ev[5].record()
+            h.cuszp_decompress_L(out.data_ptr(), cap, y.data_ptr(), n, L, ws.data_ptr(), ws.numel(), sp); ev[5].record()
             # REL chain as the product runs it: flush, range, compress (no flush between)
             flush.zero_(); ev[6].record()
             h.cuszp_range(x.data_ptr(), n, mm.data_ptr(), ws.data_ptr(), ws.numel(), sp)
-            h.cuszp_compress_minmax(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, out.data_ptr(), cap, ob.data_ptr(),
-                                    ws.data_ptr(), ws.numel(), sp); ev[7].record()
+            h.cuszp_compress_minmax_L(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, L, out.data_ptr(), cap, ob.data_ptr(),
+                                      ws.data_ptr(), ws.numel(), sp); ev[7].record()
             # REL as one call (range + compress; the library may overlap them)
             flush.zero_(); ev[8].record()
-            h.cuszp_compress(x.data_ptr(), n, a.rel, 1, out.data_ptr(), cap, ob.data_ptr(), ws.data_ptr(), ws.numel(),
-                             sp); ev[9].record()
+            h.cuszp_compress_L(x.data_ptr(), n, a.rel, 1, L, out.data_ptr(), cap, ob.data_ptr(), ws.data_ptr(),
+                               ws.numel(), sp); ev[9].record()
             torch.cuda.synchronize()
             S = int(ob.item())
             digest = (S, float(y[:1000].sum()), float(y[-1000:].sum()))

@@ -116,6 +116,7 @@ int main(int argc, char** argv) {
   for (int g : {1, 3, 4 * sms}) {
     cuszp_debug_set_grid(g, g);
     fails += round_trip(100003, 1e-4f, CUSZP_REL, 32, 1);
+    fails += round_trip(100003, 1e-4f, CUSZP_REL, 8, 1);
   }
   cuszp_debug_set_grid(0, 0);
   CK(cudaDeviceSynchronize());
