@@ -247,78 +247,53 @@ __device__ __forceinline__ uint32_t lorenzo_md_pack(uint32_t rb, int lane) {
   return (a << 1) | (uint32_t(l) >> 31);
 }
 
-// L = 8 / 16 (SL): a 32-lane row holds BR = 32 / SL blocks and a plane of a
-// block is SL / 8 BYTES (element j at byte j / 8, bit j % 8, R9
-// generalised), so a transposed word holds one plane of BR blocks: byte
-// (L = 8) or halfword (L = 16) b is block b's.  One group = 4 rows = 4 BR
-// blocks.  S rows share a transpose (S = 4 when every v < 2^8, 2 when
-// < 2^16, else 1): lane 32/S * h + k then holds plane k of row S p + h.
-//   plane counts: a ballot of "part b non-zero" over the planes of a row
-//                 segment, bit length (= F + 1, 0 for a zero block, Eq 2);
-//   offsets:      segmented scan of the block byte counts over the group;
-//   sequences:    a 4 x 4 byte (L = 8) / 2 x 2 halfword (L = 16) transpose
-//                 inside lane quads / pairs turns lane BR m + b of a segment
-//                 into bytes 4m .. 4m+3 of block b's byte sequence (sign map
-//                 then planes), stored bytewise at the block's
-//                 offset in the warp's byte ring.
-// Writes the group's packed plane counts to wb[0 .. BR-1]; returns its bytes.
-template <int SL, int S>
-__device__ __forceinline__ uint32_t place_small(const uint32_t (&v)[4], const Xpose& xpose, int lane,
-                                                uint8_t* ringb, uint32_t base, uint32_t* wb) {
-  constexpr int BR = 32 / SL, NBG = 4 * BR, NX = 4 / S, SEG = 32 / S, PB = SL / 8;
-  constexpr uint32_t kMaskB = kRing * 4 - 1;
-  uint32_t tw[NX];
-#pragma unroll
-  for (int p = 0; p < NX; ++p) {
-    const uint32_t x = (S == 4) ? pack4(v[0], v[1], v[2], v[3])
-                     : (S == 2) ? __byte_perm(v[2 * p], v[2 * p + 1], 0x5410u) : v[p];
-    tw[p] = xpose(x);
+// ---------------------------------------------------------------- L = 8 / 16
+// One L-block per LANE (thread-per-block): a plane of an L-block is L/8 BYTES
+// (element j at byte j / 8, bit j % 8, R9 generalised), so the
+// whole block -- quantisation, Lorenzo, fixed length and bit-shuffle -- runs
+// in the lane's registers and no warp transpose is needed; only the block's
+// byte offset comes from a warp scan.
+
+// 8 x 8 bit-matrix transpose of the 64-bit value hi:lo (bit p of byte i ->
+// bit i of byte p): bytes = the low / next ... byte of 8 elements -> 8 planes
+// of those elements (the block bit-shuffle), three delta swaps
+__device__ __forceinline__ void transpose8x8(uint32_t& lo, uint32_t& hi) {
+  uint32_t t;
+  t = (lo ^ (lo >> 7)) & 0x00AA00AAu;  lo ^= t ^ (t << 7);    // distance 7 and 14 stay inside
+  t = (hi ^ (hi >> 7)) & 0x00AA00AAu;  hi ^= t ^ (t << 7);    // each 32-bit half
+  t = (lo ^ (lo >> 14)) & 0x0000CCCCu; lo ^= t ^ (t << 14);
+  t = (hi ^ (hi >> 14)) & 0x0000CCCCu; hi ^= t ^ (t << 14);
+  t = (lo ^ __funnelshift_r(lo, hi, 28)) & 0xF0F0F0F0u;      // distance 28 crosses the halves
+  lo ^= t;
+  hi ^= t >> 4;
+}
+
+// byte g of 8 values -> one 64-bit row (byte i = value i's byte g)
+__device__ __forceinline__ void gather_bytes8(const uint32_t* v, uint32_t g, uint32_t& lo, uint32_t& hi) {
+  const uint32_t sel = g | ((4u + g) << 4);                     // PRMT: byte g of a, byte g of b
+  lo = __byte_perm(__byte_perm(v[0], v[1], sel), __byte_perm(v[2], v[3], sel), 0x5410u);
+  hi = __byte_perm(__byte_perm(v[4], v[5], sel), __byte_perm(v[6], v[7], sel), 0x5410u);
+}
+
+// Words 4q/W .. of an L-block's byte sequence for planes 8g .. 8g+7 (W = L/4
+// words: the sign map is plane 0, then |l| bit k-1 in plane k)
+template <int SL>
+__device__ __forceinline__ void block_seq8(const uint32_t* v, uint32_t g, uint32_t* s) {
+  uint32_t lo, hi;
+  gather_bytes8(v, g, lo, hi);
+  transpose8x8(lo, hi);
+  if constexpr (SL == 8) {
+    s[0] = lo;                                                  // planes 8g .. 8g+3, one byte each
+    s[1] = hi;
+  } else {                                                      // a plane = 2 bytes: elements 0-7, 8-15
+    uint32_t lo1, hi1;
+    gather_bytes8(v + 8, g, lo1, hi1);
+    transpose8x8(lo1, hi1);
+    s[0] = __byte_perm(lo, lo1, 0x5140u);
+    s[1] = __byte_perm(lo, lo1, 0x7362u);
+    s[2] = __byte_perm(hi, hi1, 0x5140u);
+    s[3] = __byte_perm(hi, hi1, 0x7362u);
   }
-  // plane count of block beta = lane % NBG (row beta / BR, part beta % BR)
-  const int beta = lane % NBG, row = beta / BR, part = beta % BR;
-  uint32_t bal = 0;
-#pragma unroll
-  for (int p = 0; p < NX; ++p)
-#pragma unroll
-    for (int b = 0; b < BR; ++b) {
-      const uint32_t pm = (SL == 8 ? 0xffu : 0xffffu) << (8 * PB * b);
-      const uint32_t bb = __ballot_sync(kFull, (tw[p] & pm) != 0u);
-      if (p == row / S && b == part) bal = bb;
-    }
-  const uint32_t segbits = (SEG == 32) ? bal : (bal >> (SEG * (row % S))) & ((1u << (SEG & 31)) - 1u);
-  const uint32_t planes = 32u - __clz(segbits);
-  const uint32_t bytes = planes * PB;
-  uint32_t incl = bytes;
-#pragma unroll
-  for (int o = 1; o < NBG; o <<= 1) {
-    const uint32_t y = __shfl_up_sync(kFull, incl, o, NBG);
-    if (beta >= o) incl += y;
-  }
-  const uint32_t info = (incl - bytes) | (bytes << 16);          // exclusive offset | bytes
-  const uint32_t gbytes = __shfl_sync(kFull, incl, NBG - 1);
-  uint32_t f = planes << (8 * (beta & 3));                       // 4 blocks' plane counts per word
-  f |= __shfl_xor_sync(kFull, f, 1);
-  f |= __shfl_xor_sync(kFull, f, 2);
-  if (lane < NBG && (lane & 3) == 0) wb[lane >> 2] = f;  // sync: acq_rel count, then mbarrier staged[m]
-  const int k = lane % SEG;
-  const uint32_t m = uint32_t(k / BR), b = uint32_t(k % BR);
-#pragma unroll
-  for (int p = 0; p < NX; ++p) {
-    uint32_t x = tw[p];
-    if constexpr (SL == 8) {                                     // 4 x 4 byte transpose in lane quads
-      x = __byte_perm(x, __shfl_xor_sync(kFull, x, 2), (lane & 2) ? 0x3276u : 0x5410u);
-      x = __byte_perm(x, __shfl_xor_sync(kFull, x, 1), (lane & 1) ? 0x3715u : 0x6240u);
-    } else {                                                     // 2 x 2 halfword transpose in lane pairs
-      x = __byte_perm(x, __shfl_xor_sync(kFull, x, 1), (lane & 1) ? 0x3276u : 0x5410u);
-    }
-    const uint32_t src = uint32_t(S * p + lane / SEG) * BR + b;  // block of this lane's chunk
-    const uint32_t in = __shfl_sync(kFull, info, int(src));
-    const uint32_t nb = in >> 16, pos = base + (in & 0xffffu) + 4 * m;
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-      if (4 * m + j < nb) ringb[(pos + j) & kMaskB] = uint8_t(x >> (8 * j));  // sync: ring slot freed by the writer's tail release; read after staged[m]
-  }
-  return gbytes;
 }
 
 // O = Lorenzo order: 1 (the paper's 1D 1-layer predictor) or 2 (2-layer,
@@ -336,7 +311,6 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   static_assert(SL == 0 || ((SL == 8 || SL == 16) && M == 1 && O == 1 && D == 1), "L = 8 / 16");
   constexpr bool kSmall = SL != 0;
   constexpr int kWB = kSmall ? kTileElems / SL / 4 : kTileBlocks / 4;
-  constexpr uint32_t kSegMask = (kSmall ? SL : 32) - 1;   // lane bits inside a block (Lorenzo restarts)
   extern __shared__ __align__(128) unsigned char smem_raw[];
   CompressSmem<kWB>& sm = *reinterpret_cast<CompressSmem<kWB>*>(smem_raw);
   const int lane = threadIdx.x & 31;
@@ -595,6 +569,18 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               const uint32_t hi = rw[(wi + 1) & (kRing - 1)];  // sync: ring written before staged[m] (bytes past the segment unused)
               gw[k] = __funnelshift_r(lo, hi, sh);
             }
+            // the segment's ring bytes back to zero (the compute warps OR the
+            // words they share between blocks into a zeroed ring); the words
+            // at the segment's ends are shared with the neighbouring segments
+            __syncwarp();
+            uint32_t* rz = sm.ring[w];
+            const uint32_t wa = h >> 2, nz = c ? ((h + c + 3) >> 2) - wa : 0u;
+            for (uint32_t k = lane; k < nz; k += 32) {
+              const uint32_t wi = wa + k;
+              const uint32_t lo = max(h, 4 * wi) - 4 * wi, hi = min(h + c, 4 * wi + 4) - 4 * wi;   // bytes [lo, hi)
+              if (hi - lo == 4) rz[wi & (kRing - 1)] = 0u;  // sync: copied above (syncwarp); reused after the tail release
+              else atomicAnd(&rz[wi & (kRing - 1)], ~((0xffffffffu >> (32 - 8 * (hi - lo))) << (8 * lo)));  // sync: shared word: atomic AND vs the compute warps' atomic OR
+            }
           }
         } else {
         uint32_t* dst_t = payload + excl + lane;
@@ -632,10 +618,14 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       const Xpose xpose(lane);
       // scaled-float Lorenzo (quantize_scaled2) for the paper's default L = 32, order 1
       constexpr bool kScaled = (M == 1 && O == 1 && D == 1);
-      const float kf = (uint32_t(lane) & kSegMask) ? -1.0f : -0.0f;   // -0: the lane starts a block
+      const float kf = lane ? -1.0f : -0.0f;
       const uint64_t nk = (uint64_t(__float_as_uint(kf)) << 32) | __float_as_uint(kf);
       uint32_t head = 0;                                // words this warp has appended (monotonic)
       uint32_t* ring = sm.ring[w];
+      if constexpr (kSmall) {                           // L = 8 / 16 OR shared words into a zeroed ring
+        for (uint32_t k = lane; k < kRing; k += 32) ring[k] = 0u;
+        __syncwarp();
+      }
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
@@ -670,6 +660,98 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         // group would not fit)
         uint32_t room = (kSmall ? kRing * 4 : kRing) - (head - ld_volatile_u32(&sm.tail[w]));
         uint32_t wbs[kCBPW / 4];                       // word counts of each group (bytes), for the F array
+        if constexpr (kSmall) {
+          // L = 8 / 16, one block per lane (kBPL passes of 32 blocks per tile):
+          //   a2-a4  R2 quantisation and the block Lorenzo in registers, v = 2|l| + s
+          //          (the scaled-subnormal form of quantize_scaled2, in-thread);
+          //   a5/a6  planes = bit length of the OR of v (= F + 1; 0: zero block),
+          //          c = planes * L/8 bytes (Eq 2), offsets by a warp scan;
+          //   a8     the byte sequence 8 planes at a time (gather + 8x8 bit
+          //          transpose) funnel-shifted onto 4-byte aligned ring words:
+          //          words inside the block are stored, the (<= 2) words shared
+          //          with neighbouring blocks are OR-ed into the zeroed ring.
+          constexpr int kBPL = kCBPW * 32 / SL / 32;   // 2 (L = 8), 1 (L = 16)
+          constexpr int kW = SL / 4;                   // sequence words per 8 planes
+          constexpr uint32_t kRB = kRing * 4;          // ring bytes
+          uint8_t* fcnt = reinterpret_cast<uint8_t*>(sm.meta[m].wb) + w * (kCBPW * 32 / SL);
+#pragma unroll 1
+          for (int p = 0; p < kBPL; ++p) {
+            const int blk = p * 32 + lane;
+            float x[SL];
+#pragma unroll
+            for (int q = 0; q < SL / 4; ++q) {
+              const float4 f = reinterpret_cast<const float4*>(src + blk * SL)[q];  // sync: mbarrier full[s] (TMA / producer stores); stage reused after empty[s]
+              x[4 * q] = f.x; x[4 * q + 1] = f.y; x[4 * q + 2] = f.z; x[4 * q + 3] = f.w;
+            }
+            uint32_t v[SL];
+            float resmax = 0.0f;
+            float sc_prev = 0.0f;                      // r_{-1} = 0 (scaled)
+#pragma unroll
+            for (int q = 0; q < SL / 2; ++q) {
+              const uint64_t rs = quantize_scaled2(x[2 * q], x[2 * q + 1], two_eb, recip, vmax, resmax);
+              float s0, s1;
+              asm("mov.b64 {%0, %1}, %2;" : "=f"(s0), "=f"(s1) : "l"(rs));
+              // l = r_j - r_{j-1}, exact on the subnormal grid: bits sign | |l|
+              const uint32_t l0 = __float_as_uint(__fsub_rn(s0, sc_prev));
+              const uint32_t l1 = __float_as_uint(__fsub_rn(s1, s0));
+              v[2 * q] = __funnelshift_l(l0, l0, 1);
+              v[2 * q + 1] = __funnelshift_l(l1, l1, 1);
+              sc_prev = s1;
+            }
+            if (__any_sync(kFull, resmax > eb)) {      // R2's correction somewhere in the warp: redo exactly
+              uint32_t prev = kRoundMagicBits;
+#pragma unroll
+              for (int j = 0; j < SL; ++j) {
+                const uint32_t r = quantize_exact(x[j], eb, two_eb, recip, vmax);
+                const int l = int(r - prev);
+                prev = r;
+                v[j] = (uint32_t(l < 0 ? -l : l) << 1) | (uint32_t(l) >> 31);
+              }
+            }
+            uint32_t o = 0;
+#pragma unroll
+            for (int j = 0; j < SL; ++j) o |= v[j];
+            const uint32_t planes = 32u - __clz(o);
+            fcnt[blk] = uint8_t(planes);               // sync: acq_rel count, then mbarrier staged[m]
+            wmax = max(wmax, planes);
+            const uint32_t c = planes * uint32_t(SL / 8);
+            uint32_t incl = c;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+              const uint32_t y = __shfl_up_sync(kFull, incl, d);
+              if (lane >= d) incl += y;
+            }
+            const uint32_t total = __shfl_sync(kFull, incl, 31);
+            while (cursor + total + 4 > room) {        // the pass's bytes (+ the shared word) must fit
+              room = kRB - (head - ld_volatile_u32(&sm.tail[w]));
+              if (cursor + total + 4 > room) __nanosleep(CUSZP_C_POLL_NS);
+            }
+            const uint32_t X = head + cursor + incl - c;  // ring byte of the block's first byte
+            cursor += total;
+            const uint32_t sh = 8 * (X & 3u), w0 = X >> 2;
+            const uint32_t nwords = c ? ((X & 3u) + c + 3) >> 2 : 0u;
+            const uint32_t G = (__reduce_max_sync(kFull, planes) + 7) >> 3;
+            auto emit = [&](uint32_t j, uint32_t word) {
+              uint32_t* dst = ring + ((w0 + j) & (kRing - 1));
+              if (j + 1 < nwords && j > 0) *dst = word;  // sync: ring slot freed by the writer's tail release (zeroed); read after staged[m]
+              else if (j < nwords) atomicOr(dst, word);  // sync: shared with the neighbouring blocks: atomic OR into the zeroed ring
+            };
+            uint32_t prev = 0;
+#pragma unroll
+            for (int g = 0; g < 4; ++g) {
+              if (uint32_t(g) < G) {
+                uint32_t sq[kW];
+                block_seq8<SL>(v, uint32_t(g), sq);
+#pragma unroll
+                for (int i = 0; i < kW; ++i) {
+                  emit(uint32_t(g * kW + i), __funnelshift_l(prev, sq[i], sh));
+                  prev = sq[i];
+                }
+              }
+            }
+            emit(G * kW, __funnelshift_l(prev, 0u, sh));
+          }
+        }
         // Groups of 4 blocks.  The bit transpose packs as many blocks as fit
         // in 32 bits: 4 blocks when every v < 2^8 (F <= 7), 2 when v < 2^16,
         // else 1.  After it, lane q*W + k holds word k of block q (W = 32 /
@@ -679,7 +761,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #ifdef CUSZP_DIAG_NOWORK
         for (int g = 0; g < 0; ++g) {   // diagnostics only: pipeline without the encode work
 #else
-        for (int g = 0; g < kCBPW / 4; ++g) {
+        for (int g = 0; g < (kSmall ? 0 : kCBPW / 4); ++g) {   // (L = 8 / 16: the per-lane path above)
 #endif
           float x[4];
 #pragma unroll
@@ -713,18 +795,14 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           uint32_t v[4], wq[4];
           auto counts = [&]() {
             // a5: words per block = bit length of the block's OR of v (= of its max)
-            // (L = 8 / 16: counted after the transpose, place_small)
-            if constexpr (!kSmall) {
 #pragma unroll
-              for (int q = 0; q < 4; ++q) wq[q] = 32u - __clz(__reduce_or_sync(kFull, v[q]));
-            }
+            for (int q = 0; q < 4; ++q) wq[q] = 32u - __clz(__reduce_or_sync(kFull, v[q]));
           };
           auto lorenzo_and_counts = [&]() {
             if constexpr (M == 1) {
 #pragma unroll
               for (int q = 0; q < 4; ++q)
-                v[q] = (D > 1) ? lorenzo_md_pack<D>(r[q], lane) : (O == 2) ? lorenzo2_pack(r[q], lane)
-                                                                   : lorenzo_pack(r[q], int(uint32_t(lane) & kSegMask));
+                v[q] = (D > 1) ? lorenzo_md_pack<D>(r[q], lane) : (O == 2) ? lorenzo2_pack(r[q], lane) : lorenzo_pack(r[q], lane);
             } else {
               // a block continues across its sub-blocks: lane 0 of sub-block q
               // takes lane 31 of sub-block q-1 unless q starts a block
@@ -752,91 +830,75 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             lorenzo_and_counts();
           }
 #endif
-          if constexpr (kSmall) {
-            const uint32_t span = 32u - __clz(__reduce_or_sync(kFull, v[0] | v[1] | v[2] | v[3]));
-            wmax = max(wmax, span);
-            // room for a worst-case group (4 BR blocks x 32 planes x SL/8 bytes = 512 bytes)
-            while (cursor + 512 > room) {
-              room = kRing * 4 - (head - ld_volatile_u32(&sm.tail[w]));
-              if (cursor + 512 > room) __nanosleep(CUSZP_C_POLL_NS);
-            }
-            uint8_t* ringb = reinterpret_cast<uint8_t*>(ring);
-            uint32_t* wbg = &sm.meta[m].wb[(w * (kCBPW / 4) + g) * (32 / SL)];
-            const uint32_t base = head + cursor;
-            if (span <= 8) cursor += place_small<SL, 4>(v, xpose, lane, ringb, base, wbg);
-            else if (span <= 16) cursor += place_small<SL, 2>(v, xpose, lane, ringb, base, wbg);
-            else cursor += place_small<SL, 1>(v, xpose, lane, ringb, base, wbg);
-          } else {
-            // room in this warp's ring for a worst-case group (4 x 32 words)
-            while (cursor + 4 * 32 > room) {
-              room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
-              if (cursor + 4 * 32 > room) __nanosleep(CUSZP_C_POLL_NS);
-            }
-            if constexpr (M == 2) {                                        // one F per block
-              wq[0] = wq[1] = max(wq[0], wq[1]);
-              wq[2] = wq[3] = max(wq[2], wq[3]);
-            } else if constexpr (M == 4) {
-              wq[0] = wq[1] = wq[2] = wq[3] = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
-            }
-            // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
-            // flagged ERANGE at the end.  Such garbage blocks still take at most
-            // 32 words (v is 32-bit), which the capacity bound covers (DESIGN 9.5).
-            const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
-            wmax = max(wmax, span);
-            const uint32_t wb = pack4(wq[0], wq[1], wq[2], wq[3]);
-            const uint32_t base = head + cursor;
-            if (M > 1) {
-              // word k of sub-block q -> block payload position M k + q % M
-              const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
-              if (span <= 8) {
-                const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
-                const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
-                const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
-                if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-              } else if (span <= 16) {
-                const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
-                const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
-                const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
-                if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-                const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
-                const uint32_t sub23 = (M == 2) ? h : 2u + h;
-                if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-              } else {
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                  const uint32_t tq = xpose(v[q]);
-                  const uint32_t pre = (q & ~(M - 1)) == 0 ? 0u : __byte_perm(pb, 0, 0x4440u + (q & ~(M - 1)));
-                  if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-                }
-              }
-            } else if (span <= 8) {
+          // room in this warp's ring for a worst-case group (4 x 32 words)
+          while (cursor + 4 * 32 > room) {
+            room = kRing - (head - ld_volatile_u32(&sm.tail[w]));
+            if (cursor + 4 * 32 > room) __nanosleep(CUSZP_C_POLL_NS);
+          }
+          if constexpr (M == 2) {                                        // one F per block
+            wq[0] = wq[1] = max(wq[0], wq[1]);
+            wq[2] = wq[3] = max(wq[2], wq[3]);
+          } else if constexpr (M == 4) {
+            wq[0] = wq[1] = wq[2] = wq[3] = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+          }
+          // > 25 words only for data failing the R5 guard (NaN/Inf, |r0| >= 2^23):
+          // flagged ERANGE at the end.  Such garbage blocks still take at most
+          // 32 words (v is 32-bit), which the capacity bound covers (DESIGN 9.5).
+          const uint32_t span = max(max(wq[0], wq[1]), max(wq[2], wq[3]));
+          wmax = max(wmax, span);
+          const uint32_t wb = pack4(wq[0], wq[1], wq[2], wq[3]);
+          const uint32_t base = head + cursor;
+          if (M > 1) {
+            // word k of sub-block q -> block payload position M k + q % M
+            const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
+            if (span <= 8) {
               const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
-              const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
-              const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
-              if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              const uint32_t q = uint32_t(lane) >> 3, k = lane & 7;
+              const uint32_t pre = __byte_perm(pb, 0, 0x4440u + (q & ~uint32_t(M - 1)));
+              if (k < __byte_perm(wb, 0, 0x4440u + q)) ring[(base + pre + M * k + (q & (M - 1))) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             } else if (span <= 16) {
               const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
               const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
-              const bool hi = lane >= 16;
-              const uint32_t k = lane & 15;
-              if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-              if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              const uint32_t h = lane >= 16 ? 1u : 0u, k = lane & 15;
+              if (k < wq[0]) ring[(base + M * k + h) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              const uint32_t pre23 = (M == 2) ? wq[0] + wq[1] : 0u;
+              const uint32_t sub23 = (M == 2) ? h : 2u + h;
+              if (k < wq[2]) ring[(base + pre23 + M * k + sub23) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             } else {
-              uint32_t o = base;
 #pragma unroll
               for (int q = 0; q < 4; ++q) {
                 const uint32_t tq = xpose(v[q]);
-                if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
-                o += wq[q];
+                const uint32_t pre = (q & ~(M - 1)) == 0 ? 0u : __byte_perm(pb, 0, 0x4440u + (q & ~(M - 1)));
+                if (uint32_t(lane) < wq[q]) ring[(base + pre + M * uint32_t(lane) + (q & (M - 1))) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
               }
             }
-            cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
-#if CUSZP_C_GUNROLL >= 4
-            wbs[g] = wb;
-#else
-            if (lane == 0) sm.meta[m].wb[w * (kCBPW / 4) + g] = wb;  // sync: acq_rel count, then mbarrier staged[m]
-#endif
+          } else if (span <= 8) {
+            const uint32_t tw = xpose(pack4(v[0], v[1], v[2], v[3]));
+            const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
+            const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
+            if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+          } else if (span <= 16) {
+            const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
+            const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
+            const bool hi = lane >= 16;
+            const uint32_t k = lane & 15;
+            if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+            if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+          } else {
+            uint32_t o = base;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const uint32_t tq = xpose(v[q]);
+              if (uint32_t(lane) < wq[q]) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+              o += wq[q];
+            }
           }
+          cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
+#if CUSZP_C_GUNROLL >= 4
+          wbs[g] = wb;
+#else
+          if (lane == 0) sm.meta[m].wb[w * (kCBPW / 4) + g] = wb;  // sync: acq_rel count, then mbarrier staged[m]
+#endif
         }
         __syncwarp();
         if (lane == 0) {
@@ -844,7 +906,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           TileMeta<kWB>& md = sm.meta[m];
           // the group word counts go to the writer, which stores the tile's F bytes
 #if CUSZP_C_GUNROLL >= 4
-          if constexpr (kSmall) {}
+          if constexpr (kSmall) {}                       // F bytes stored per block (small path)
           else if constexpr (kCBPW / 4 == 4) *reinterpret_cast<uint4*>(&md.wb[w * 4]) = make_uint4(wbs[0], wbs[1], wbs[2], wbs[3]);  // sync: acq_rel count, then mbarrier staged[m]; slot reused after released
           else *reinterpret_cast<uint2*>(&md.wb[w * 2]) = make_uint2(wbs[0], wbs[1]);  // sync: acq_rel count, then mbarrier staged[m]
 #endif

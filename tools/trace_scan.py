@@ -38,6 +38,9 @@ def load(path):
     h.cuszp_max_compressed_bytes.argtypes = [sz]
     h.cuszp_max_compressed_bytes.restype = sz
     h.cuszp_debug_set_trace.argtypes = [vp]
+    h.cuszp_compress_minmax_L.argtypes = [vp, sz, f32, vp, i32, i32, vp, sz, vp, vp, sz, vp]
+    h.cuszp_max_compressed_bytes_L.argtypes = [sz, i32]
+    h.cuszp_max_compressed_bytes_L.restype = sz
     return h
 
 
@@ -88,6 +91,7 @@ def main():
     ap.add_argument("--config", default="c2_hurricane")
     ap.add_argument("--rel", type=float, default=1e-2)
     ap.add_argument("--field", default=None)
+    ap.add_argument("--L", type=int, default=32, help="block length; L != 32 traces compression only")
     a = ap.parse_args()
     import synth
 
@@ -97,7 +101,7 @@ def main():
     n = x.numel()
     nt = ((n + 31) // 32 + 127) // 128
     ws = torch.zeros(h.cuszp_workspace_bytes(n), dtype=torch.uint8, device=dev)
-    cap = h.cuszp_max_compressed_bytes(n)
+    cap = h.cuszp_max_compressed_bytes_L(n, a.L)
     out = torch.empty(cap, dtype=torch.uint8, device=dev)
     ob = torch.zeros(1, dtype=torch.int64, device=dev)
     mm = torch.empty(2, dtype=torch.float32, device=dev)
@@ -112,19 +116,26 @@ def main():
         flush.zero_()
         h.cuszp_range(x.data_ptr(), n, mm.data_ptr(), ws.data_ptr(), ws.numel(), sp)
         ev[0].record()
-        h.cuszp_compress_minmax(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, out.data_ptr(), cap, ob.data_ptr(),
-                                ws.data_ptr(), ws.numel(), sp)
+        h.cuszp_compress_minmax_L(x.data_ptr(), n, a.rel, mm.data_ptr(), 1, a.L, out.data_ptr(), cap, ob.data_ptr(),
+                                  ws.data_ptr(), ws.numel(), sp)
         ev[1].record()
         if traced:
             torch.cuda.synchronize()
             trc = trace[: nt * 8].view(nt, 8).cpu().numpy().astype(np.int64)
             trace.zero_()
             trace[: nt * 8].view(nt, 8)[:, 4] = (1 << 62)
+        if a.L != 32:
+            continue
         flush.zero_()
         ev[2].record()
         h.cuszp_decompress(out.data_ptr(), cap, y.data_ptr(), n, ws.data_ptr(), ws.numel(), sp)
         torch.cuda.synchronize()
     h.cuszp_debug_set_trace(None)
+    if a.L != 32:
+        S = int(ob.item())
+        print(f"n={n} tiles={nt} S={S} CR={4 * n / S:.2f} L={a.L}  compress {ev[0].elapsed_time(ev[1]) * 1e3:.1f} us")
+        report("compress", trc, ev[0].elapsed_time(ev[1]) * 1e6)
+        return
     trd = trace[: nt * 8].view(nt, 8).cpu().numpy().astype(np.int64)
     pw = trace[nt * 8:nt * 16].view(nt, 8).cpu().numpy().astype(np.int64)
     pk = trace[nt * 16:].view(nt, 8).cpu().numpy().astype(np.int64)
