@@ -569,18 +569,6 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               const uint32_t hi = rw[(wi + 1) & (kRing - 1)];  // sync: ring written before staged[m] (bytes past the segment unused)
               gw[k] = __funnelshift_r(lo, hi, sh);
             }
-            // the segment's ring bytes back to zero (the compute warps OR the
-            // words they share between blocks into a zeroed ring); the words
-            // at the segment's ends are shared with the neighbouring segments
-            __syncwarp();
-            uint32_t* rz = sm.ring[w];
-            const uint32_t wa = h >> 2, nz = c ? ((h + c + 3) >> 2) - wa : 0u;
-            for (uint32_t k = lane; k < nz; k += 32) {
-              const uint32_t wi = wa + k;
-              const uint32_t lo = max(h, 4 * wi) - 4 * wi, hi = min(h + c, 4 * wi + 4) - 4 * wi;   // bytes [lo, hi)
-              if (hi - lo == 4) rz[wi & (kRing - 1)] = 0u;  // sync: copied above (syncwarp); reused after the tail release
-              else atomicAnd(&rz[wi & (kRing - 1)], ~((0xffffffffu >> (32 - 8 * (hi - lo))) << (8 * lo)));  // sync: shared word: atomic AND vs the compute warps' atomic OR
-            }
           }
         } else {
         uint32_t* dst_t = payload + excl + lane;
@@ -622,10 +610,6 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       const uint64_t nk = (uint64_t(__float_as_uint(kf)) << 32) | __float_as_uint(kf);
       uint32_t head = 0;                                // words this warp has appended (monotonic)
       uint32_t* ring = sm.ring[w];
-      if constexpr (kSmall) {                           // L = 8 / 16 OR shared words into a zeroed ring
-        for (uint32_t k = lane; k < kRing; k += 32) ring[k] = 0u;
-        __syncwarp();
-      }
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
@@ -726,15 +710,26 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               room = kRB - (head - ld_volatile_u32(&sm.tail[w]));
               if (cursor + total + 4 > room) __nanosleep(CUSZP_C_POLL_NS);
             }
+            // zero the pass's ring words ahead of the OR-ed shared words (all but
+            // a first word shared with the previous pass, whose later bytes are
+            // zero already)
+            {
+              const uint32_t B = head + cursor, E = B + total;
+              for (uint32_t k = ((B + 3) >> 2) + lane; k < ((E + 3) >> 2); k += 32) ring[k & (kRing - 1)] = 0u;  // sync: free ring space (room checked); own warp's words
+              __syncwarp();
+            }
             const uint32_t X = head + cursor + incl - c;  // ring byte of the block's first byte
             cursor += total;
             const uint32_t sh = 8 * (X & 3u), w0 = X >> 2;
             const uint32_t nwords = c ? ((X & 3u) + c + 3) >> 2 : 0u;
             const uint32_t G = (__reduce_max_sync(kFull, planes) + 7) >> 3;
+            // word j of the block (aligned ring word w0 + j): words 1 .. nwords-2
+            // lie inside the block and are stored; word 0 and word nwords-1 may
+            // share bytes with the neighbouring blocks and are OR-ed in at the end
+            uint32_t first = 0, last = 0;
             auto emit = [&](uint32_t j, uint32_t word) {
-              uint32_t* dst = ring + ((w0 + j) & (kRing - 1));
-              if (j + 1 < nwords && j > 0) *dst = word;  // sync: ring slot freed by the writer's tail release (zeroed); read after staged[m]
-              else if (j < nwords) atomicOr(dst, word);  // sync: shared with the neighbouring blocks: atomic OR into the zeroed ring
+              if (j + 1 < nwords) ring[(w0 + j) & (kRing - 1)] = word;  // sync: ring slot freed by the writer's tail release (zeroed); read after staged[m]
+              last = (j + 1 == nwords) ? word : last;
             };
             uint32_t prev = 0;
 #pragma unroll
@@ -744,12 +739,20 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
                 block_seq8<SL>(v, uint32_t(g), sq);
 #pragma unroll
                 for (int i = 0; i < kW; ++i) {
-                  emit(uint32_t(g * kW + i), __funnelshift_l(prev, sq[i], sh));
+                  const uint32_t word = __funnelshift_l(prev, sq[i], sh);
+                  if (g == 0 && i == 0) {
+                    first = word;
+                    last = nwords == 1 ? word : 0u;
+                  } else {
+                    emit(uint32_t(g * kW + i), word);
+                  }
                   prev = sq[i];
                 }
               }
             }
-            emit(G * kW, __funnelshift_l(prev, 0u, sh));
+            if (G) emit(G * kW, __funnelshift_l(prev, 0u, sh));
+            if (nwords) atomicOr(ring + (w0 & (kRing - 1)), first);  // sync: shared with the previous block(s): atomic OR into the zeroed ring
+            if (nwords > 1) atomicOr(ring + ((w0 + nwords - 1) & (kRing - 1)), last);  // sync: shared with the next block(s): atomic OR into the zeroed ring
           }
         }
         // Groups of 4 blocks.  The bit transpose packs as many blocks as fit
