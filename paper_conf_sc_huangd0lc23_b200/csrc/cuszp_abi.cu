@@ -14,7 +14,8 @@ namespace {
 uint64_t num_blocks(uint64_t n, int L = kL) { return (n + L - 1) / L; }
 // M = L / 32 for the block lengths of SURVEY 8(f) rank 3 (0: unsupported)
 int sub_blocks(int L) { return L == 32 ? 1 : L == 64 ? 2 : L == 128 ? 4 : 0; }
-int mi(int M) { return M == 1 ? 0 : M == 2 ? 1 : 2; }
+// index of a block length in the per-L occupancy tables (8, 16, 32, 64, 128)
+int lidx(int L) { return L == 8 ? 0 : L == 16 ? 1 : L == 32 ? 2 : L == 64 ? 3 : 4; }
 // L = 8 / 16: byte-granular planes, the one-thread-per-block path (small_l.cu)
 bool small_L(int L) { return L == 8 || L == 16; }
 bool valid_L(int L) { return sub_blocks(L) != 0 || small_L(L); }
@@ -24,7 +25,7 @@ struct DeviceInfo {
   int sms = 0;
   int occ_compress = 0, occ_decompress = 0, occ_range = 0, occ_quality = 0;
   int occ_c[5] = {0, 0, 0, 0, 0};   // compress, per L = 8, 16, 32, 64, 128
-  int occ_d[3] = {0, 0, 0};         // decompress, per M = 1, 2, 4
+  int occ_d[5] = {0, 0, 0, 0, 0};   // decompress, per L = 8, 16, 32, 64, 128
 };
 
 // Per-device launch geometry, computed once: persistent grids of
@@ -41,13 +42,13 @@ int device_info(DeviceInfo* out) {
     if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return CUSZP_ECUDA;
     for (int k = 0; k < 5; ++k)
       if (compress_configure(8 << k, &d.occ_c[k]) != cudaSuccess) return CUSZP_ECUDA;
-    for (int k = 0; k < 3; ++k)
-      if (decompress_configure(1 << k, &d.occ_d[k]) != cudaSuccess) return CUSZP_ECUDA;
+    for (int k = 0; k < 5; ++k)
+      if (decompress_configure(8 << k, &d.occ_d[k]) != cudaSuccess) return CUSZP_ECUDA;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_range, range_kernel, 256, 0) != cudaSuccess ||
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ_quality, quality_kernel, 256, 0) != cudaSuccess)
       return CUSZP_ECUDA;
     d.occ_compress = d.occ_c[2];
-    d.occ_decompress = d.occ_d[0];
+    d.occ_decompress = d.occ_d[2];
     cache[dev] = d;
     have[dev] = true;
   }
@@ -137,7 +138,7 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   // diagnostics build: the three-launch L = 8 / 16 path (small_l.cu), for A/B
   if (small_L(L)) return compress_small_launch(L, a, stream) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 #endif
-  const int occ = di.occ_c[L == 8 ? 0 : L == 16 ? 1 : 2 + mi(M)];
+  const int occ = di.occ_c[lidx(L)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_compress > 0) grid = uint64_t(g_grid_compress);
   if (grid > a.num_tiles) grid = a.num_tiles;
@@ -310,17 +311,20 @@ int cuszp_decompress_ex(const void* d_in, size_t in_bytes, float* d_out, size_t 
   a.nx = n;
   a.nby = 1;
   a.nbx = a.nb;
+#ifdef CUSZP_SMALL_L_3PASS
+  // diagnostics build: the three-launch L = 8 / 16 path (small_l.cu), for A/B
   if (small_L(block_len))
     return decompress_small_launch(block_len, a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK
                                                                                                 : CUSZP_ECUDA;
-  const int occ = di.occ_d[mi(M)];
+#endif
+  const int occ = di.occ_d[lidx(block_len)];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);
   a.chunk_tiles = decompress_chunk_tiles(a.num_tiles, grid);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  return decompress_launch(M, order, unsigned(grid), a, s) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
+  return decompress_launch(block_len, order, unsigned(grid), a, s) == cudaSuccess ? CUSZP_OK : CUSZP_ECUDA;
 }
 
 size_t cuszp_num_blocks_md(size_t nz, size_t ny, size_t nx, int dims) {
@@ -396,13 +400,13 @@ int cuszp_decompress_md(const void* d_in, size_t in_bytes, float* d_out, size_t 
   a.nx = g.nx;
   a.nby = g.nby;
   a.nbx = g.nbx;
-  const int occ = di.occ_d[0];
+  const int occ = di.occ_d[2];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);
   a.chunk_tiles = decompress_chunk_tiles(a.num_tiles, grid);
   if (grid > a.num_tiles) grid = a.num_tiles;
   if (grid < 1) grid = 1;
-  return decompress_launch(1, 1, unsigned(grid), a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK
+  return decompress_launch(32, 1, unsigned(grid), a, static_cast<cudaStream_t>(stream)) == cudaSuccess ? CUSZP_OK
                                                                                                     : CUSZP_ECUDA;
 }
 

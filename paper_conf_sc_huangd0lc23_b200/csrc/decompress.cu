@@ -61,14 +61,18 @@ struct ChunkDesc {
   uint32_t ntiles;
 };
 
+// FB = bytes of fixed-length (F) bytes staged per tile: 512 / 256 for
+// L = 8 / 16 (one F per block, read by the lane that decodes the block)
+template <int FB>
 struct DecompressSmem {
-  uint32_t data[kDStages][kDataWords];         // 51.3 KB
+  uint32_t data[kDStages][kDataWords];         // 25.7 KB
   uint2 ginfo[kDStages][kGroups];              // per 4-block group: {words per block (bytes), offset | mode << 16}
   uint32_t tile[kDStages];
   uint32_t delta[kDStages];                    // first payload word of the tile inside data[]
   ChunkDesc chunk[2];
   alignas(16) uint32_t scratch[kComputeWarps][4 * 32];   // per-warp transposed rows of one group
   uint64_t full[kDStages];                     // TMA completion (the only mbarriers)
+  alignas(16) uint8_t fbytes[kDStages][FB];
 };
 
 // named barriers (id 0 is __syncthreads)
@@ -76,6 +80,50 @@ constexpr uint32_t kBarEmpty0 = 1;
 constexpr uint32_t kBarReady0 = kBarEmpty0 + kDStages, kBarFree0 = kBarReady0 + 2;
 constexpr uint32_t kBarCount = 32 + 32 * kComputeWarps;   // loader + compute warps
 static_assert(kBarFree0 + 2 <= 16, "named barriers");
+
+// 8 x 8 bit-matrix transpose of hi:lo (bit p of byte i -> bit i of byte p),
+// self-inverse: 8 planes of 8 elements -> the elements' bytes (a10 for
+// L = 8 / 16; the compressor's transpose8x8)
+__device__ __forceinline__ void untranspose8x8(uint32_t& lo, uint32_t& hi) {
+  uint32_t t;
+  t = (lo ^ (lo >> 7)) & 0x00AA00AAu;  lo ^= t ^ (t << 7);
+  t = (hi ^ (hi >> 7)) & 0x00AA00AAu;  hi ^= t ^ (t << 7);
+  t = (lo ^ (lo >> 14)) & 0x0000CCCCu; lo ^= t ^ (t << 14);
+  t = (hi ^ (hi >> 14)) & 0x0000CCCCu; hi ^= t ^ (t << 14);
+  t = (lo ^ __funnelshift_r(lo, hi, 28)) & 0xF0F0F0F0u;
+  lo ^= t;
+  hi ^= t >> 4;
+}
+
+// byte e of hi:lo -> byte g of v[e] (8 byte permutes)
+template <int G>
+__device__ __forceinline__ void scatter_bytes8(uint32_t lo, uint32_t hi, uint32_t* v) {
+  constexpr uint32_t kKeep = 0x3210u & ~(0xFu << (4 * G));
+#pragma unroll
+  for (int e = 0; e < 8; ++e)
+    v[e] = __byte_perm(v[e], e < 4 ? lo : hi, kKeep | ((4u + uint32_t(e & 3)) << (4 * G)));
+}
+
+// planes 8g .. 8g+7 of an L-block's byte sequence (kW = L/4 words) -> byte g
+// of each element's v = 2|l| + s (inverse of the compressor's block_seq8)
+template <int SL>
+__device__ __forceinline__ void block_unseq8(const uint32_t* sq, int g, uint32_t* v) {
+  auto put = [&](uint32_t lo, uint32_t hi, uint32_t* ve) {
+    untranspose8x8(lo, hi);
+    switch (g) {
+      case 0: scatter_bytes8<0>(lo, hi, ve); break;
+      case 1: scatter_bytes8<1>(lo, hi, ve); break;
+      case 2: scatter_bytes8<2>(lo, hi, ve); break;
+      default: scatter_bytes8<3>(lo, hi, ve); break;
+    }
+  };
+  if constexpr (SL == 8) {
+    put(sq[0], sq[1], v);
+  } else {                                          // plane = [elements 0-7 byte, elements 8-15 byte]
+    put(__byte_perm(sq[0], sq[1], 0x6420u), __byte_perm(sq[2], sq[3], 0x6420u), v);
+    put(__byte_perm(sq[0], sq[1], 0x7531u), __byte_perm(sq[2], sq[3], 0x7531u), v + 8);
+  }
+}
 
 }  // namespace
 
@@ -86,15 +134,19 @@ static_assert(kBarFree0 + 2 <= 16, "named barriers");
 // 1x4x8 / 2x4x4 blocks and scatter each block's rows into the (nz, ny, nx) field.
 // CT = tiles per look-back chunk (4 or 8; 8 is instantiated for the main path
 // only, chosen by the host for large inputs).
-template <int M, int O, int D = 1, int CT = 4>
+// SL = 8 / 16: byte-granular block lengths, one block per lane (M = 1).
+template <int M, int O, int D = 1, int CT = 4, int SL = 0>
 __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kernel(DecompressArgs a) {
   static_assert(CT == 4 || CT == 8, "chunk of 4 or 8 tiles");
+  static_assert(SL == 0 || ((SL == 8 || SL == 16) && M == 1 && O == 1 && D == 1), "L = 8 / 16");
+  constexpr bool kSmall = SL != 0;
+  constexpr int kFT = kSmall ? kTileElems / SL : 16;            // F bytes per tile (L = 8 / 16)
   static_assert(D == 1 || (M == 1 && O == 1), "multi-dimensional Lorenzo with L = 32, order 1");
   static_assert(M == 1 || M == 2 || M == 4, "L in {32, 64, 128}");
   static_assert(O == 1 || (O == 2 && M == 1), "2-layer Lorenzo with L = 32");
-  constexpr uint32_t kLog2L = 5 + (M == 2 ? 1 : M == 4 ? 2 : 0);
+  constexpr uint32_t kLog2L = SL == 8 ? 3 : SL == 16 ? 4 : 5 + (M == 2 ? 1 : M == 4 ? 2 : 0);
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  DecompressSmem& sm = *reinterpret_cast<DecompressSmem*>(smem_raw);
+  DecompressSmem<kFT>& sm = *reinterpret_cast<DecompressSmem<kFT>*>(smem_raw);
   const int lane = threadIdx.x & 31;
   const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);   // provably warp-uniform (no divergence checks before warp-sync ops)
   pdl_wait();                                     // compression / previous call complete
@@ -122,8 +174,8 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
     else if (a.n > 0) {
       const float two = __fadd_rn(eb, eb);
       if (!(eb >= kFltMin) || !isfinite(two)) err = CUSZP_ECORRUPT;
-      else if ((pbytes & 3u) || a.in_bytes < p0 || a.in_bytes - p0 < pbytes) err = CUSZP_ECORRUPT;
-      payload_words = pbytes / 4;
+      else if ((!kSmall && (pbytes & 3u)) || a.in_bytes < p0 || a.in_bytes - p0 < pbytes) err = CUSZP_ECORRUPT;
+      payload_words = kSmall ? pbytes : pbytes / 4;        // look-back unit: bytes for L = 8 / 16
     }
   }
   const float two_eb = __fadd_rn(eb, eb);
@@ -160,6 +212,82 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 #ifdef CUSZP_TRACE
         if (a.trace && uint32_t(lane) < ntiles) trace_put(a.trace, t0 + lane, 0, global_ns());
 #endif
+        if constexpr (kSmall) {
+          // L = 8 / 16: lane L sums the block bytes (Eq 2: (F + 1) L/8, 0 for
+          // F = 0) of kSPL warp slices of the chunk (slice q = tile q / 8,
+          // compute warp q % 8; 64 / 32 F bytes each, 16 per load).
+          constexpr int kSlice = kFT / kComputeWarps;
+          constexpr int kSPL = CT * kComputeWarps / 32;         // slices per lane: 2 (CT = 8) or 1
+          constexpr int kLPT = kComputeWarps / kSPL;            // lanes per tile
+          uint32_t ssum[kSPL], fmax = 0, lsum = 0;
+#pragma unroll
+          for (int h = 0; h < kSPL; ++h) {
+            const uint32_t q = uint32_t(kSPL * lane + h);
+            const uint64_t blk0 = uint64_t(t0 + q / 8) * kFT + (q % 8) * kSlice;
+            uint4 f[kSlice / 16];
+#pragma unroll
+            for (int k = 0; k < kSlice / 16; ++k) {             // all loads in flight first
+              const uint64_t bk = blk0 + 16 * k;
+              f[k] = bk < a.nb ? *reinterpret_cast<const uint4*>(a.in + kHdr + bk) : make_uint4(0, 0, 0, 0);
+            }
+            uint32_t sum = 0;
+#pragma unroll
+            for (int k = 0; k < kSlice / 16; ++k) {
+              const uint64_t bk = blk0 + 16 * k;
+              uint32_t x[4] = {f[k].x, f[k].y, f[k].z, f[k].w};
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                if (bk + 4 * e + 4 > a.nb) {                    // the F area's padding: zero blocks
+                  const int keep = int(a.nb > bk + 4 * e ? a.nb - bk - 4 * e : 0);
+                  x[e] &= __funnelshift_rc(0xffffffffu, 0u, uint32_t(32 - 8 * keep));
+                }
+                fmax = __vmaxu4(fmax, x[e]);
+                const uint32_t y = x[e] + (__vcmpne4(x[e], 0u) & 0x01010101u);   // F + 1 or 0 per byte
+                sum += (y * 0x01010101u) >> 24;                 // <= 4 x 25
+              }
+            }
+            ssum[h] = sum * uint32_t(SL / 8);
+            lsum += ssum[h];
+          }
+          // tile-local exclusive slice offsets: segmented scan over a tile's lanes
+          uint32_t incl = lsum;
+#pragma unroll
+          for (int o = 1; o < kLPT; o <<= 1) incl = uint32_t(scan_step_up(int(incl), o, (32 - kLPT) << 8));
+          uint32_t ttot[CT], tpre[CT], agg = 0;
+#pragma unroll
+          for (int k = 0; k < CT; ++k) {
+            ttot[k] = __shfl_sync(kFull, incl, kLPT * k + kLPT - 1);
+            tpre[k] = agg;
+            agg += ttot[k];
+          }
+          const bool badf = __any_sync(kFull, __vcmpgtu4(fmax, 0x18181818u) != 0u);   // F > 24
+          if (lane == 0) publish_aggregate(a.status, c, agg, epoch);
+          const uint64_t excl = resolve_prefix(a.status, c, agg, epoch);
+          const bool oob = badf || excl + agg > payload_words;  // decode zeros, never read past in_bytes
+          if (oob) bad |= kBadCorrupt;
+          const int tl = lane / kLPT;
+          uint32_t off = incl - lsum;
+#pragma unroll
+          for (int h = 0; h < kSPL; ++h) {
+            cd.gmeta[tl][(kSPL * lane + h) % 8] = oob ? 0xffffffffu : off;   // 0xffffffff: a zero tile
+            off += ssum[h];
+          }
+          uint64_t ts = 0;
+          uint32_t tw = 0;
+#pragma unroll
+          for (int k = 0; k < CT; ++k)
+            if (lane == k) { ts = excl + tpre[k]; tw = oob ? 0u : ttot[k]; }
+          if (lane < CT) {
+            cd.tile_start[lane] = ts;
+            cd.tile_words[lane] = tw;
+          }
+          if (lane == 0) {
+            cd.chunk = c;
+            cd.ntiles = ntiles;
+          }
+          named_arrive(kBarReady0 + b, 64);
+          continue;
+        }
         // The chunk in parts of 4 tiles (ct / 4 of them): in part h, lane L takes
         // sub-blocks 16L .. 16L+15 of tiles 4h .. 4h+3 = groups 4(L%8) .. +3 of
         // tile 4h + L/8 = blocks (16L ..)/M.  All F loads of the chunk are
@@ -296,23 +424,35 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           uint32_t tma_bytes = 0, delta = 0;
           uint64_t a0 = 0;
           if (tw > 0) {
-            const uint64_t start = p0 + 4 * cd.tile_start[j], end = start + 4 * tw;
+            constexpr uint32_t kU = kSmall ? 1u : 4u;             // bytes per look-back unit
+            const uint64_t start = p0 + kU * cd.tile_start[j], end = start + kU * tw;
             a0 = start & ~uint64_t(15);
             uint64_t a1 = (end + 15) & ~uint64_t(15);
             if (a1 > a.in_bytes) a1 = a.in_bytes & ~uint64_t(15);
             tma_bytes = uint32_t(a1 - a0);
-            delta = uint32_t(start - a0) / 4;
-            // words past the last full 16 bytes inside in_bytes (<= 3)
-            const uint64_t tail_words = end > a1 ? (end - a1) / 4 : 0;
-            if (uint64_t(lane) < tail_words)
-              sm.data[s][(a1 - a0) / 4 + lane] = *reinterpret_cast<const uint32_t*>(a.in + a1 + 4 * lane);  // sync: mbarrier full[s]
+            delta = uint32_t(start - a0) / kU;
+            if constexpr (kSmall) {
+              // bytes past the last full 16 bytes inside in_bytes (<= 15)
+              const uint64_t tail = end > a1 ? end - a1 : 0;
+              if (uint64_t(lane) < tail)
+                reinterpret_cast<uint8_t*>(sm.data[s])[(a1 - a0) + lane] = a.in[a1 + lane];  // sync: mbarrier full[s]
+            } else {
+              // words past the last full 16 bytes inside in_bytes (<= 3)
+              const uint64_t tail_words = end > a1 ? (end - a1) / 4 : 0;
+              if (uint64_t(lane) < tail_words)
+                sm.data[s][(a1 - a0) / 4 + lane] = *reinterpret_cast<const uint32_t*>(a.in + a1 + 4 * lane);  // sync: mbarrier full[s]
+            }
           }
           __syncwarp();
           if (lane == 0) {
             sm.tile[s] = cd.chunk * ct + j;  // sync: mbarrier full[s]
             sm.delta[s] = delta;  // sync: mbarrier full[s]
-            mbar_arrive_expect_tx(&sm.full[s], tma_bytes);   // one phase per use, even with 0 bytes
+            // L = 8 / 16: the tile's F bytes too (the decoding lanes read them)
+            const uint32_t t_ld = cd.chunk * ct + j;
+            const uint32_t fb = kSmall ? uint32_t(min(uint64_t(kFT), align16(a.nb) - uint64_t(t_ld) * kFT)) : 0u;
+            mbar_arrive_expect_tx(&sm.full[s], tma_bytes + fb);   // one phase per use, even with 0 bytes
             if (tma_bytes) tma_load_1d(sm.data[s], a.in + a0, tma_bytes, &sm.full[s]);
+            if (kSmall) tma_load_1d(sm.fbytes[s], a.in + kHdr + uint64_t(t_ld) * kFT, fb, &sm.full[s]);
 #ifdef CUSZP_TRACE
             trace_put(a.trace, cd.chunk * ct + j, 3, global_ns());
             trace_put(a.trace, cd.chunk * ct + j, 7, blockIdx.x);
@@ -321,6 +461,100 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
           ++k;
         }
         named_arrive(kBarFree0 + b, 64);
+      }
+    } else if constexpr (kSmall) {
+      // ------------------------------------------- compute, L = 8 / 16
+      // One block per lane (kBPL passes of 32 blocks per tile): the lane's F
+      // byte gives its planes (F + 1, 0 for a zero block) and bytes (Eq 2); a
+      // warp scan plus the scanner's slice offset places the block in the
+      // staged payload; its byte sequence is read as funnel-shifted words
+      // (bytes past the block masked off), 8 planes at a time turned back
+      // into element bytes by the self-inverse 8x8 bit transpose (a10), then
+      // the in-register prefix sum (a11) and dequantisation (a12).
+      const int w = warp - kDFirstCompute;
+      constexpr int kSlice = kFT / kComputeWarps;
+      constexpr int kBPL = kSlice / 32;                            // 2 (L = 8), 1 (L = 16)
+      constexpr int kW = SL / 4;                                    // sequence words per 8 planes
+      const float two_eb_s = __fmul_rn(two_eb, 0x1p23f);
+      const bool scaled_ok = isfinite(two_eb_s);
+      for (uint32_t i = 0;; ++i) {
+        const int s = int(i % kDStages);
+        mbar_wait(&sm.full[s], (i / kDStages) & 1u);            // payload + F bytes landed
+        const uint32_t t = sm.tile[s];  // sync: mbarrier full[s]
+        if (t == kSentinel) break;
+        const uint32_t so_raw = sm.ginfo[s][w].y;  // sync: mbarrier full[s]
+        const bool zero_tile = so_raw == 0xffffffffu;
+        uint32_t base = sm.delta[s] + (zero_tile ? 0u : so_raw);  // sync: mbarrier full[s]
+#pragma unroll 1
+        for (int p = 0; p < kBPL; ++p) {
+          const uint32_t blk = uint32_t(p * 32 + lane);                // block in the warp's slice
+          const uint64_t gblk = uint64_t(t) * kFT + uint64_t(w) * kSlice + blk;
+          uint32_t F = sm.fbytes[s][w * kSlice + blk];  // sync: mbarrier full[s]
+          if (gblk >= a.nb || zero_tile || F > uint32_t(kMaxF)) F = 0;
+          const uint32_t planes = F ? F + 1 : 0u, c = planes * uint32_t(SL / 8);
+          uint32_t incl = c;
+#pragma unroll
+          for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, incl, d);
+            if (lane >= d) incl += y;
+          }
+          const uint32_t off = base + incl - c;                      // byte offset in data[s]
+          base += __shfl_sync(kFull, incl, 31);
+          const uint32_t G = (__reduce_max_sync(kFull, planes) + 7) >> 3;
+          const uint32_t* dw = sm.data[s] + (off >> 2);
+          const uint32_t sh = 8 * (off & 3u);
+          uint32_t v[SL];
+#pragma unroll
+          for (int e = 0; e < SL; ++e) v[e] = 0;
+          uint32_t wprev = dw[0];  // sync: mbarrier full[s]
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            if (uint32_t(g) < G) {
+              uint32_t sq[kW];
+#pragma unroll
+              for (int k = 0; k < kW; ++k) {
+                const int j = g * kW + k;
+                const uint32_t wn = dw[j + 1];  // sync: mbarrier full[s]
+                const int rem = int(c) - 4 * j;                      // bytes of the block left
+                sq[k] = __funnelshift_r(wprev, wn, sh) &
+                        __funnelshift_rc(0xffffffffu, 0u, uint32_t(min(max(32 - 8 * rem, 0), 32)));
+                wprev = wn;
+              }
+              block_unseq8<SL>(sq, g, v);
+            }
+          }
+          float* o = a.out + uint64_t(t) * kTileElems + uint64_t(w) * (kSlice * SL) + uint64_t(blk) * SL;
+          float d[SL];
+          if (scaled_ok) {
+            // v rotated right by one = sign | |l|: the subnormal l * 2^-149;
+            // the running sum is exact (|r| < 2^23), then (r 2^-149 * 2^126) *
+            // (2eb * 2^23) is the single rounding of r * 2eb (R13)
+            float r = 0.0f;
+#pragma unroll
+            for (int e = 0; e < SL; ++e) {
+              r = __fadd_rn(r, __uint_as_float(__funnelshift_r(v[e], v[e], 1)));
+              d[e] = __fmul_rn(__fmul_rn(r, 0x1p126f), two_eb_s);
+            }
+          } else {
+            int r = 0;
+#pragma unroll
+            for (int e = 0; e < SL; ++e) {
+              r += (v[e] & 1u) ? -int(v[e] >> 1) : int(v[e] >> 1);
+              d[e] = __fmul_rn(__int2float_rn(r), two_eb);
+            }
+          }
+          const uint64_t i0 = uint64_t(o - a.out);
+          if (i0 + SL <= a.n) {
+#pragma unroll
+            for (int q = 0; q < SL / 4; ++q)
+              reinterpret_cast<float4*>(o)[q] = make_float4(d[4 * q], d[4 * q + 1], d[4 * q + 2], d[4 * q + 3]);
+          } else {
+#pragma unroll
+            for (int e = 0; e < SL; ++e)
+              if (i0 + e < a.n) o[e] = d[e];
+          }
+        }
+        named_arrive(kBarEmpty0 + s, kBarCount);
       }
     } else {
       // ------------------------------------------------------------ compute
@@ -621,44 +855,63 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
 }
 
 namespace {
-template <int M, int O = 1, int D = 1, int CT = 4>
+template <int M, int O = 1, int D = 1, int CT = 4, int SL = 0>
 cudaError_t configure_m(int* occ) {
-  const int smem = int(sizeof(DecompressSmem));
-  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O, D, CT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O, D, CT>, kDThreads, smem);
+  constexpr int kFT = SL ? kTileElems / SL : 16;
+  const int smem = int(sizeof(DecompressSmem<kFT>));
+  cudaError_t e = cudaFuncSetAttribute(decompress_kernel<M, O, D, CT, SL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, decompress_kernel<M, O, D, CT, SL>, kDThreads, smem);
   return e;
+}
+template <int M, int O = 1, int D = 1, int CT = 4, int SL = 0>
+cudaError_t launch_k(cudaLaunchConfig_t cfg, const DecompressArgs& a) {
+  constexpr int kFT = SL ? kTileElems / SL : 16;
+  cfg.dynamicSmemBytes = sizeof(DecompressSmem<kFT>);
+  return cudaLaunchKernelEx(&cfg, decompress_kernel<M, O, D, CT, SL>, a);
 }
 }  // namespace
 
-cudaError_t decompress_configure(int M, int* occ) {
+// L in {8, 16, 32, 64, 128}: resident CTAs per SM of that block length's kernel
+cudaError_t decompress_configure(int L, int* occ) {
   int occ2 = 0;
-  if (M == 1 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
-                 configure_m<1, 1, 3>(&occ2) != cudaSuccess || configure_m<1, 1, 1, 8>(&occ2) != cudaSuccess))
+  if (L == 32 && (configure_m<1, 2>(&occ2) != cudaSuccess || configure_m<1, 1, 2>(&occ2) != cudaSuccess ||
+                  configure_m<1, 1, 3>(&occ2) != cudaSuccess || configure_m<1, 1, 1, 8>(&occ2) != cudaSuccess))
     return cudaErrorUnknown;
-  return M == 1 ? configure_m<1>(occ) : M == 2 ? configure_m<2>(occ) : configure_m<4>(occ);
+  if (L == 8 && configure_m<1, 1, 1, 8, 8>(&occ2) != cudaSuccess) return cudaErrorUnknown;
+  if (L == 16 && configure_m<1, 1, 1, 8, 16>(&occ2) != cudaSuccess) return cudaErrorUnknown;
+  switch (L) {
+    case 8: return configure_m<1, 1, 1, 4, 8>(occ);
+    case 16: return configure_m<1, 1, 1, 4, 16>(occ);
+    case 32: return configure_m<1>(occ);
+    case 64: return configure_m<2>(occ);
+    default: return configure_m<4>(occ);
+  }
 }
 
-cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s) {
+cudaError_t decompress_launch(int L, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kDThreads);
-  cfg.dynamicSmemBytes = sizeof(DecompressSmem);
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;   // see pdl_wait()
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (a.dims == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 2>, a);
-  if (a.dims == 3) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 3>, a);
-  if (order == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 2>, a);
-  if (M == 1 && a.chunk_tiles == 8) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1, 1, 8>, a);
-  if (M == 1) return cudaLaunchKernelEx(&cfg, decompress_kernel<1, 1>, a);
-  if (M == 2) return cudaLaunchKernelEx(&cfg, decompress_kernel<2, 1>, a);
-  return cudaLaunchKernelEx(&cfg, decompress_kernel<4, 1>, a);
+  const bool c8 = a.chunk_tiles == 8;
+  if (a.dims == 2) return launch_k<1, 1, 2>(cfg, a);
+  if (a.dims == 3) return launch_k<1, 1, 3>(cfg, a);
+  if (order == 2) return launch_k<1, 2>(cfg, a);
+  switch (L) {
+    case 8: return c8 ? launch_k<1, 1, 1, 8, 8>(cfg, a) : launch_k<1, 1, 1, 4, 8>(cfg, a);
+    case 16: return c8 ? launch_k<1, 1, 1, 8, 16>(cfg, a) : launch_k<1, 1, 1, 4, 16>(cfg, a);
+    case 32: return c8 ? launch_k<1, 1, 1, 8>(cfg, a) : launch_k<1, 1>(cfg, a);
+    case 64: return launch_k<2, 1>(cfg, a);
+    default: return launch_k<4, 1>(cfg, a);
+  }
 }
 
-size_t decompress_smem_bytes() { return sizeof(DecompressSmem); }
+size_t decompress_smem_bytes() { return sizeof(DecompressSmem<16>); }
 int decompress_threads() { return kDThreads; }
 
 }  // namespace cuszp

@@ -470,8 +470,8 @@ constexpr int kQualityMaxGrid = 2048;
 // defined next to them (compress.cu / decompress.cu): M in {1, 2, 4}.
 cudaError_t compress_configure(int L, int* occupancy);        // smem attribute + CTAs per SM (L = block length)
 cudaError_t compress_launch(int L, int order, unsigned grid, const CompressArgs& a, cudaStream_t s);
-cudaError_t decompress_configure(int M, int* occupancy);
-cudaError_t decompress_launch(int M, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s);
+cudaError_t decompress_configure(int L, int* occupancy);
+cudaError_t decompress_launch(int L, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s);
 // L in {8, 16} (small_l.cu): three launches each, one thread per L-block.
 cudaError_t compress_small_launch(int L, const CompressArgs& a, cudaStream_t s);
 cudaError_t decompress_small_launch(int L, const DecompressArgs& a, cudaStream_t s);
