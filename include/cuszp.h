@@ -127,7 +127,8 @@ int cuszp_decompress(const void* d_in, size_t in_bytes, float* d_out, size_t n,
  * need cuszp_max_compressed_bytes_L(n, L) bytes (32 + align16(nb) +
  * 32 L/8 nb, nb = ceil(n/L)); workspaces are sized as for L = 32.
  * block_len outside {8, 16, 32, 64, 128}: EINVAL (the size helper returns 0).
- * L = 8 / 16 run three launches per call (csrc/small_l.cu); same statuses.
+ * L = 8 / 16 run the same one-pass kernels with byte-granular placement
+ * (a plane is 1 / 2 bytes; one block per lane); same statuses.
  * Decompression must be given the stream's L (a header with another L:
  * async ECORRUPT). */
 size_t cuszp_max_compressed_bytes_L(size_t n, int block_len);

@@ -472,7 +472,8 @@ cudaError_t compress_configure(int L, int* occupancy);        // smem attribute 
 cudaError_t compress_launch(int L, int order, unsigned grid, const CompressArgs& a, cudaStream_t s);
 cudaError_t decompress_configure(int L, int* occupancy);
 cudaError_t decompress_launch(int L, int order, unsigned grid, const DecompressArgs& a, cudaStream_t s);
-// L in {8, 16} (small_l.cu): three launches each, one thread per L-block.
+// L in {8, 16}, diagnostics build only (-DCUSZP_SMALL_L_3PASS, small_l.cu): the
+// round-1 three-launch path, the A/B baseline of the one-pass kernels.
 cudaError_t compress_small_launch(int L, const CompressArgs& a, cudaStream_t s);
 cudaError_t decompress_small_launch(int L, const DecompressArgs& a, cudaStream_t s);
 __global__ void quality_kernel(QualityArgs a);

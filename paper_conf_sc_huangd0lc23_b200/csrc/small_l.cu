@@ -1,22 +1,21 @@
-// small_l.cu -- block lengths L in {8, 16} (the
-// paper's smoothness analysis spans L = 8..128, Fig 6).
+// small_l.cu -- DIAGNOSTICS ONLY (built with -DCUSZP_SMALL_L_3PASS): the
+// round-1 three-launch path for block lengths L in {8, 16}, kept as the A/B
+// baseline of the one-pass kernels (compress.cu / decompress.cu, SL = 8 / 16,
+// DESIGN 9.4).  The production library does not contain these kernels.
 //
-// At L <= 16 a bit plane is one or two BYTES (R9 generalised),
-// so the word-granular warp transpose of the L >= 32 kernels does not
-// apply.  This path is one thread per L-block, tiles of 4096 elements
-// (the L = 32 tile, so the caller's workspace holds one u64 per tile):
+// One thread per L-block, tiles of 4096 elements:
 //   compress:   sizes (quantise, Lorenzo, F, tile byte sums)  ->
 //               tile scan + header (one CTA)                   ->
 //               write (re-quantise, CTA scan of block bytes, sign map + planes)
 //   decompress: sizes (F -> tile byte sums) -> tile scan + header check ->
 //               decode (CTA scan, planes -> |l|, signs, prefix sum, r * 2eb)
-// Three launches each and the input is read twice on compress: a correct
-// first path for the variant, not a tuned one (DESIGN 9.4).
 //
 // Status words: each tile's byte sum / exclusive prefix is stored < 2^40,
-// so its epoch field is 0 and the look-back of the L >= 32 kernels (epochs
-// >= 1) never takes it for a published word.
+// so its epoch field is 0 and the look-back of the persistent kernels
+// (epochs >= 1) never takes it for a published word.
 #include "internal.cuh"
+
+#ifdef CUSZP_SMALL_L_3PASS
 
 namespace cuszp {
 namespace {
@@ -474,3 +473,5 @@ cudaError_t decompress_small_launch(int L, const DecompressArgs& a, cudaStream_t
 }
 
 }  // namespace cuszp
+
+#endif  // CUSZP_SMALL_L_3PASS
