@@ -57,6 +57,9 @@ namespace {
 #ifndef CUSZP_C_GUNROLL
 #define CUSZP_C_GUNROLL 4
 #endif
+#ifndef CUSZP_C_FULL_POLL_NS
+#define CUSZP_C_FULL_POLL_NS 0   // > 0: compute warps poll their input stage with test + nanosleep
+#endif
 constexpr int kGUnroll = CUSZP_C_GUNROLL;         // groups of 4 blocks unrolled in the encode loop
 constexpr int kStages = CUSZP_C_STAGES;          // input ring depth (16 KB tiles)
 constexpr int kWriters = CUSZP_C_WRITERS;        // scan + writer warps
@@ -613,7 +616,19 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       for (uint32_t i = 0;; ++i) {
         const int s = int(i % kStages);
         const int m = int(i % kMeta);
+#if CUSZP_C_FULL_POLL_NS > 0
+        // test + sleep: try_wait's suspension wakes on unrelated barrier
+        // traffic (~40 re-tries per wait measured), each re-try costing issue slots
+        if (!mbar_test(&sm.full[s], (i / kStages) & 1u)) {
+          uint32_t ns = CUSZP_C_FULL_POLL_NS;
+          do {
+            __nanosleep(ns);
+            ns = min(2 * ns, 1024u);
+          } while (!mbar_test(&sm.full[s], (i / kStages) & 1u));
+        }
+#else
         mbar_wait(&sm.full[s], (i / kStages) & 1u);         // suspending wait: no issue slots taken
+#endif
         const uint32_t t = sm.in_tile[s];  // sync: mbarrier full[s]
 #ifdef CUSZP_TRACE
         // (diagnostics build only: a lane-0 branch here makes ptxas treat the

@@ -132,3 +132,39 @@ def test_small_L_interleaved_with_word_kernels_and_corrupt_F():
     y = cz.decompress(out, x_np.size, in_bytes=int(nb.item()), block_len=8)
     assert cz.last_status() == cz.OK
     assert torch.max(torch.abs(y - x)).item() <= float(cz.read_header(out)["eb_abs"]) * 1.001
+
+
+@pytest.mark.parametrize("Lb", [8, 16])
+def test_small_L_corrupt_and_truncated_streams(Lb):
+    """L = 8 / 16 streams are byte-granular (payload sizes need not be a
+    multiple of 4): a stream cut by 1..3 bytes, F above 24, F bytes that
+    disagree with the header's payload size and random byte flips must only
+    ever give a status; the workspace keeps working afterwards."""
+    rng = np.random.default_rng(Lb)
+    n = 70_001
+    x_np = np.cumsum(rng.standard_normal(n)).astype(np.float32)
+    x = torch.from_numpy(x_np).to(DEV)
+    ws = cz.Workspace(n)
+    out, nb = cz.compress(x, 1e-3, "rel", block_len=Lb, ws=ws)
+    S = int(nb.item())
+    y = torch.empty(n, device=DEV)
+    for cut in (1, 2, 3, 17):
+        cz.decompress(out, n, out=y, in_bytes=S - cut, ws=ws, block_len=Lb)
+        assert cz.last_status(ws) == cz.ECORRUPT, cut
+    c = out.clone(); c[32 + 7] = 25                                  # F > 24
+    cz.decompress(c, n, out=y, in_bytes=S, ws=ws, block_len=Lb)
+    assert cz.last_status(ws) == cz.ECORRUPT
+    c = out.clone(); c[32 + 9] = (int(c[32 + 9]) + 1) % 25           # sizes disagree with the header
+    cz.decompress(c, n, out=y, in_bytes=S + 400, ws=ws, block_len=Lb)
+    assert cz.last_status(ws) == cz.ECORRUPT
+    nbk = (n + Lb - 1) // Lb
+    for _ in range(40):
+        c = out.clone()
+        for p in rng.integers(0, 32 + nbk, 3):
+            c[int(p)] = int(rng.integers(0, 256))
+        cz.decompress(c, n, out=y, in_bytes=S, ws=ws, block_len=Lb)
+        assert cz.last_status(ws) in (cz.OK, cz.ECORRUPT, cz.EINVAL, cz.ERANGE)
+    cz.decompress(out, n, out=y, in_bytes=S, ws=ws, block_len=Lb)
+    assert cz.last_status(ws) == cz.OK
+    st, y_o = oracle.decompress(out[:S].cpu().numpy(), n)
+    assert st == oracle.OK and np.array_equal(y.cpu().numpy().view(np.uint32), y_o.view(np.uint32))

@@ -82,6 +82,20 @@ static int round_trip(size_t n, float eb, int mode, int L, int order) {
     CK(cudaMemcpy(&h, d_exact, 32, cudaMemcpyDeviceToHost));
     bad = (st != CUSZP_OK);
   }
+  if (!bad && S > 33) {
+    // a stream cut by one byte, in an exact-size allocation: ECORRUPT, no read past it
+    void* d_cut = nullptr;
+    CK(cudaMalloc(&d_cut, S - 1));
+    CK(cudaMemcpy(d_cut, d_out, S - 1, cudaMemcpyDeviceToDevice));
+    OKS(cuszp_decompress_ex(d_cut, S - 1, d_y, n, L, order, d_ws, wsb, nullptr));
+    if (cuszp_last_status(d_ws, nullptr) != CUSZP_ECORRUPT) {
+      std::fprintf(stderr, "n=%zu L=%d order=%d: truncated stream not ECORRUPT\n", n, L, order);
+      bad = 1;
+    }
+    CK(cudaFree(d_cut));
+    OKS(cuszp_decompress_ex(d_exact, S, d_y, n, L, order, d_ws, wsb, nullptr));   // the full stream again
+    CK(cudaMemcpy(y.data(), d_y, n * sizeof(float), cudaMemcpyDeviceToHost));
+  }
   for (size_t i = 0; i < n && !bad; ++i) {
     const double ulp = double(std::nextafterf(std::fabs(x[i]), INFINITY)) - std::fabs(double(x[i]));
     if (std::fabs(double(x[i]) - double(y[i])) > double(h.eb_abs) + ulp) {
