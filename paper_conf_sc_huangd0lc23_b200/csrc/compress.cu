@@ -395,38 +395,39 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         }
         const uint32_t dst0 = smem_u32(sm.in[s]);
         // lane l gathers blocks l, l+32, l+64, l+96 of the tile (neighbouring
-        // lanes read neighbouring row segments); block coordinates from one
-        // 32-bit division per block (nb < 2^32, checked on the host)
+        // lanes read neighbouring row segments); block coordinates by
+        // multiply-shift division (FastDiv; nb < 2^32, checked on the host),
+        // row r of the block at a compile-time (z, y, x) step from its origin
+        const uint64_t plane = a.ny * a.nx;
 #pragma unroll 1
         for (uint32_t ib = lane; ib < uint32_t(kTileBlocks); ib += 32) {
           const uint32_t b = t * uint32_t(kTileBlocks) + ib;
           const uint32_t nbx = uint32_t(a.nbx), nby = uint32_t(a.nby);
-          const uint32_t kyz = b / nbx, kx = b - kyz * nbx;
-          const uint32_t kz = kyz / nby, ky = kyz - kz * nby;
+          const uint32_t kyz = a.fd_nbx.div(b), kx = b - kyz * nbx;
+          const uint32_t kz = a.fd_nby.div(kyz), ky = kyz - kz * nby;
           const bool blk_in = uint64_t(b) < a.nb;
+          const uint64_t z0 = uint64_t(kz) * (D == 3 ? 2 : 1), y0 = uint64_t(ky) * 4;
+          const uint64_t x0 = uint64_t(kx) * (D == 3 ? 4 : 8);
+          const float* org = a.in + (blk_in ? z0 * plane + y0 * a.nx + x0 : 0);
+          const uint32_t dst_b = dst0 + 4u * (ib * 32u);
 #pragma unroll
           for (uint32_t r = 0; r < 8; ++r) {                          // the block's 8 row segments of 4 points
-            uint64_t gz, gy, gx;
-            uint32_t d;                                                // element index in the block
-            if constexpr (D == 2) {
-              gz = kz; gy = uint64_t(ky) * 4 + (r >> 1); gx = uint64_t(kx) * 8 + 4 * (r & 1u);
-              d = (r >> 1) * 8 + 4 * (r & 1u);
-            } else {
-              gz = uint64_t(kz) * 2 + (r >> 2); gy = uint64_t(ky) * 4 + (r & 3u); gx = uint64_t(kx) * 4;
-              d = r * 4;
-            }
-            const bool row_in = blk_in && gz < a.nz && gy < a.ny;
-            const float* src = a.in + (row_in ? (gz * a.ny + gy) * a.nx + gx : 0);
-            const uint32_t dst = dst0 + 4u * (ib * 32u + d);
+            // 2D: row r/2, x half r%2 (element (r/2)*8 + 4(r%2)); 3D: z r/4, y r%4 (element 4r)
+            const uint32_t rz = (D == 3) ? (r >> 2) : 0u, ry = (D == 3) ? (r & 3u) : (r >> 1);
+            const uint32_t rx = (D == 3) ? 0u : 4u * (r & 1u);
+            const uint32_t d = (D == 3) ? r * 4 : (r >> 1) * 8 + 4 * (r & 1u);
+            const bool row_in = blk_in && z0 + rz < a.nz && y0 + ry < a.ny;
+            const float* src = org + (rz ? plane : 0) + ry * a.nx + rx;
+            const uint32_t dst = dst_b + 4u * d;
             if (al16) {
-              const uint32_t bytes = (row_in && gx < a.nx) ? 16u : 0u;   // nx % 4 == 0: a row of 4 is all in or all out
+              const uint32_t bytes = (row_in && x0 + rx < a.nx) ? 16u : 0u;   // nx % 4 == 0: a row of 4 is all in or all out
               asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(bytes ? src : a.in),
                            "r"(bytes)
                            : "memory");
             } else {
 #pragma unroll
               for (int e = 0; e < 4; ++e) {
-                const uint32_t bytes = (row_in && gx + e < a.nx) ? 4u : 0u;
+                const uint32_t bytes = (row_in && x0 + rx + e < a.nx) ? 4u : 0u;
                 asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(dst + 4 * e),
                              "l"(bytes ? src + e : a.in), "r"(bytes)
                              : "memory");

@@ -124,6 +124,10 @@ int launch_compress(const float* d_in, size_t n, int mode, float eb_in, const fl
   a.nx = md ? md->nx : n;
   a.nby = md ? md->nby : 1;
   a.nbx = md ? md->nbx : nb;
+  if (md) {
+    a.fd_nbx = FastDiv(uint32_t(md->nbx));
+    a.fd_nby = FastDiv(uint32_t(md->nby));
+  }
   a.mode = mode;
   a.eb_in = eb_in;
   a.minmax = d_minmax;
@@ -400,6 +404,8 @@ int cuszp_decompress_md(const void* d_in, size_t in_bytes, float* d_out, size_t 
   a.nx = g.nx;
   a.nby = g.nby;
   a.nbx = g.nbx;
+  a.fd_nbx = FastDiv(uint32_t(g.nbx));
+  a.fd_nby = FastDiv(uint32_t(g.nby));
   const int occ = di.occ_d[2];
   uint64_t grid = uint64_t(di.sms) * uint64_t(occ > 0 ? occ : 1);
   if (g_grid_decompress > 0) grid = uint64_t(g_grid_decompress);

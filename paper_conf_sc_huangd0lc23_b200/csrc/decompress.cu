@@ -751,8 +751,8 @@ __global__ void __launch_bounds__(kDThreads, CUSZP_D_MINBLOCKS) decompress_kerne
             dd[2] = __fmul_rn(__int2float_rn(e2), two_eb);
             dd[3] = __fmul_rn(__int2float_rn(e3), two_eb);
             const uint32_t b = t * uint32_t(kTileBlocks) + uint32_t(w) * kBPW + uint32_t(g) * 4u + q;
-            const uint32_t kx = b % uint32_t(a.nbx), kyz = b / uint32_t(a.nbx);
-            const uint32_t ky = kyz % uint32_t(a.nby), kz = kyz / uint32_t(a.nby);
+            const uint32_t kyz = a.fd_nbx.div(b), kx = b - kyz * uint32_t(a.nbx);   // FastDiv (internal.cuh)
+            const uint32_t kz = a.fd_nby.div(kyz), ky = kyz - kz * uint32_t(a.nby);
             uint64_t gz, gy, gx;
             if constexpr (D == 2) { gz = kz; gy = ky * 4u + (k8 >> 1); gx = kx * 8u + 4u * (k8 & 1u); }
             else { gz = kz * 2u + (k8 >> 2); gy = ky * 4u + (k8 & 3u); gx = kx * 4u; }

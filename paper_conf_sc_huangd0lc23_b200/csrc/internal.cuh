@@ -412,6 +412,26 @@ __device__ __forceinline__ void finish_call(WsCtrl* ws, uint64_t* status, uint32
 }
 
 // ------------------------------------------------------------ kernel params
+// Division by a launch-invariant 32-bit divisor d >= 1 (Granlund-Montgomery,
+// round-up multiplier): q = (t + ((n - t) >> s1)) >> s2, t = umulhi(n, m),
+// exact for every 32-bit n.  The multi-dimensional block coordinates use it
+// instead of a ~20-instruction integer division per block.
+struct FastDiv {
+  uint32_t m = 1, s1 = 0, s2 = 0;
+  FastDiv() = default;
+  __host__ explicit FastDiv(uint32_t d) {
+    uint32_t l = 0;
+    while (l < 32 && (uint64_t(1) << l) < d) ++l;                     // ceil(log2 d)
+    m = uint32_t(((uint64_t(1) << 32) * ((uint64_t(1) << l) - d)) / d + 1);
+    s1 = l < 1 ? l : 1;
+    s2 = l > 1 ? l - 1 : 0;
+  }
+  __device__ __forceinline__ uint32_t div(uint32_t n) const {
+    const uint32_t t = __umulhi(n, m);
+    return (t + ((n - t) >> s1)) >> s2;
+  }
+};
+
 struct CompressArgs {
   const float* in;
   uint64_t n;
@@ -430,6 +450,7 @@ struct CompressArgs {
   int dims;                  // Lorenzo dimensions (R18): 1, or 2 / 3 over the (nz, ny, nx) field below
   uint64_t nz, ny, nx;       // field shape (dims > 1; n = nz ny nx)
   uint64_t nby, nbx;         // block grid rows / columns (dims > 1; nb = nbz nby nbx)
+  FastDiv fd_nbx, fd_nby;    // division by nbx / nby (dims > 1)
 };
 
 struct DecompressArgs {
@@ -446,6 +467,7 @@ struct DecompressArgs {
   int dims;                  // as CompressArgs
   uint64_t nz, ny, nx;
   uint64_t nby, nbx;
+  FastDiv fd_nbx, fd_nby;
   uint32_t chunk_tiles;      // tiles per look-back chunk: 8 for large inputs, 4 for small ones (balance)
 };
 
