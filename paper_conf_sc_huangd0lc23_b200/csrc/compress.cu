@@ -299,6 +299,26 @@ __device__ __forceinline__ void block_seq8(const uint32_t* v, uint32_t g, uint32
   }
 }
 
+// lorenzo_md_pack on SCALED values (quantize_scaled2's r 2^-149): the
+// successive differences along x, y (and z) are exact subtractions on the
+// subnormal grid while they stay below 2^23 -- always under the R18 guards
+// (|r| < 2^21 in 2D, 2^20 in 3D); the result's bits are sign | |l| and a
+// rotate gives v.  Data failing a guard give garbage v (flagged ERANGE).
+template <int D>
+__device__ __forceinline__ uint32_t lorenzo_md_scaled(float rs, int lane) {
+  constexpr int kBX = (D == 3) ? 4 : 8;
+  const float px = __shfl_up_sync(kFull, rs, 1);
+  float l = (lane % kBX) ? __fsub_rn(rs, px) : rs;            // along x
+  const float uy = __shfl_up_sync(kFull, l, kBX);
+  if ((lane / kBX) % 4) l = __fsub_rn(l, uy);                 // along y
+  if constexpr (D == 3) {
+    const float uz = __shfl_up_sync(kFull, l, 16);
+    if (lane >= 16) l = __fsub_rn(l, uz);                     // along z
+  }
+  const uint32_t b = __float_as_uint(l);
+  return __funnelshift_l(b, b, 1);
+}
+
 // O = Lorenzo order: 1 (the paper's 1D 1-layer predictor) or 2 (2-layer,
 // SURVEY 8(f) rank 4; L = 32 only).
 // D = Lorenzo dimensions (DESIGN R18): 1 = the paper's 1D
@@ -609,7 +629,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       const int w = warp - kFirstCompute;
       const Xpose xpose(lane);
       // scaled-float Lorenzo (quantize_scaled2) for the paper's default L = 32, order 1
-      constexpr bool kScaled = (M == 1 && O == 1 && D == 1);
+      constexpr bool kScaled = (M == 1 && O == 1);       // L = 32, order 1, any dimensions
       const float kf = lane ? -1.0f : -0.0f;
       const uint64_t nk = (uint64_t(__float_as_uint(kf)) << 32) | __float_as_uint(kf);
       uint32_t head = 0;                                // words this warp has appended (monotonic)
@@ -836,8 +856,16 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             counts();
           };
           if constexpr (kScaled) {
-            lorenzo_scaled2(rs01, nk, v[0], v[1]);
-            lorenzo_scaled2(rs23, nk, v[2], v[3]);
+            if constexpr (D == 1) {
+              lorenzo_scaled2(rs01, nk, v[0], v[1]);
+              lorenzo_scaled2(rs23, nk, v[2], v[3]);
+            } else {
+              float f[4];
+              asm("mov.b64 {%0, %1}, %2;" : "=f"(f[0]), "=f"(f[1]) : "l"(rs01));
+              asm("mov.b64 {%0, %1}, %2;" : "=f"(f[2]), "=f"(f[3]) : "l"(rs23));
+#pragma unroll
+              for (int q = 0; q < 4; ++q) v[q] = lorenzo_md_scaled<D>(f[q], lane);
+            }
             counts();
           } else {
             lorenzo_and_counts();
