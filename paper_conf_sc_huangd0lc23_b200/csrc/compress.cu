@@ -57,6 +57,9 @@ namespace {
 #ifndef CUSZP_C_GUNROLL
 #define CUSZP_C_GUNROLL 4
 #endif
+#ifndef CUSZP_C_L2_AHEAD
+#define CUSZP_C_L2_AHEAD 1       // > 0: prefetch the input tile this many grids ahead into L2
+#endif
 #ifndef CUSZP_C_FULL_POLL_NS
 #define CUSZP_C_FULL_POLL_NS 0   // > 0: compute warps poll their input stage with test + nanosleep
 #endif
@@ -205,6 +208,14 @@ __device__ __forceinline__ uint32_t lorenzo_pack_first(uint32_t rb, int lane, ui
   const int l = int(rb - prev);
   const uint32_t a = uint32_t(l < 0 ? -l : l);
   return (a << 1) | (uint32_t(l) >> 31);
+}
+
+// bit length of x (0 for x = 0): bfind gives the index of the highest set bit
+// or 0xffffffff, so one add ends it (32 - clz compiles to FLO + two adds)
+__device__ __forceinline__ uint32_t bitlen(uint32_t x) {
+  uint32_t p;
+  asm("bfind.u32 %0, %1;" : "=r"(p) : "r"(x));
+  return p + 1u;
 }
 
 // bytes a, b, c, d (each < 256) -> one word, as 3 byte permutes
@@ -490,6 +501,17 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           for (uint32_t k = tma_bytes / 4; k < ne; ++k) sm.in[s][k] = a.in[e0 + k];   // <= 3 tail floats  // sync: mbarrier full[s] (the producer's arrive.expect_tx releases them)
           mbar_arrive_expect_tx(&sm.full[s], tma_bytes);
           if (tma_bytes) tma_load_1d(sm.in[s], a.in + e0, tma_bytes, &sm.full[s]);
+#if CUSZP_C_L2_AHEAD > 0
+          {
+            // a third input stage in L2: tickets advance about one grid per
+            // round, so the tile CUSZP_C_L2_AHEAD grids ahead is taken (by
+            // some CTA) that much later and its TMA then hits L2
+            const uint64_t tp = uint64_t(t) + uint64_t(CUSZP_C_L2_AHEAD) * gridDim.x;
+            if (tp * kTileElems + kTileElems <= a.n)
+              asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a.in + tp * kTileElems), "r"(uint32_t(kTileElems * 4))
+                           : "memory");
+          }
+#endif
         }
       }
 
@@ -731,7 +753,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             uint32_t o = 0;
 #pragma unroll
             for (int j = 0; j < SL; ++j) o |= v[j];
-            const uint32_t planes = 32u - __clz(o);
+            const uint32_t planes = bitlen(o);
             fcnt[blk] = uint8_t(planes);               // sync: acq_rel count, then mbarrier staged[m]
             wmax = max(wmax, planes);
             const uint32_t c = planes * uint32_t(SL / 8);
@@ -835,7 +857,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           auto counts = [&]() {
             // a5: words per block = bit length of the block's OR of v (= of its max)
 #pragma unroll
-            for (int q = 0; q < 4; ++q) wq[q] = 32u - __clz(__reduce_or_sync(kFull, v[q]));
+            for (int q = 0; q < 4; ++q) wq[q] = bitlen(__reduce_or_sync(kFull, v[q]));
           };
           auto lorenzo_and_counts = [&]() {
             if constexpr (M == 1) {
