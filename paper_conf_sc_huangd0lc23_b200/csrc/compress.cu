@@ -712,75 +712,86 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           //          transpose) funnel-shifted onto 4-byte aligned ring words:
           //          words inside the block are stored, the (<= 2) words shared
           //          with neighbouring blocks are OR-ed into the zeroed ring.
-          constexpr int kBPL = kCBPW * 32 / SL / 32;   // 2 (L = 8), 1 (L = 16)
+          // each lane encodes the 16 consecutive floats 16 l .. 16 l + 15 of the
+          // warp's 512-element slice: kBL = 2 blocks at L = 8, 1 at L = 16
+          constexpr int kBL = 16 / SL;
           constexpr int kW = SL / 4;                   // sequence words per 8 planes
           constexpr uint32_t kRB = kRing * 4;          // ring bytes
           uint8_t* fcnt = reinterpret_cast<uint8_t*>(sm.meta[m].wb) + w * (kCBPW * 32 / SL);
-#pragma unroll 1
-          for (int p = 0; p < kBPL; ++p) {
-            const int blk = p * 32 + lane;
-            float x[SL];
+          float x[16];
 #pragma unroll
-            for (int q = 0; q < SL / 4; ++q) {
-              const float4 f = reinterpret_cast<const float4*>(src + blk * SL)[q];  // sync: mbarrier full[s] (TMA / producer stores); stage reused after empty[s]
-              x[4 * q] = f.x; x[4 * q + 1] = f.y; x[4 * q + 2] = f.z; x[4 * q + 3] = f.w;
-            }
-            uint32_t v[SL];
-            float resmax = 0.0f;
-            float sc_prev = 0.0f;                      // r_{-1} = 0 (scaled)
+          for (int q = 0; q < 4; ++q) {
+            const float4 f = reinterpret_cast<const float4*>(src + 16 * lane)[q];  // sync: mbarrier full[s] (TMA / producer stores); stage reused after empty[s]
+            x[4 * q] = f.x; x[4 * q + 1] = f.y; x[4 * q + 2] = f.z; x[4 * q + 3] = f.w;
+          }
+          uint32_t v[16];
+          float resmax = 0.0f;
+          float sc_prev = 0.0f;                        // r_{-1} = 0 (scaled) at each block start
 #pragma unroll
-            for (int q = 0; q < SL / 2; ++q) {
-              const uint64_t rs = quantize_scaled2(x[2 * q], x[2 * q + 1], two_eb, recip, vmax, resmax);
-              float s0, s1;
-              asm("mov.b64 {%0, %1}, %2;" : "=f"(s0), "=f"(s1) : "l"(rs));
-              // l = r_j - r_{j-1}, exact on the subnormal grid: bits sign | |l|
-              const uint32_t l0 = __float_as_uint(__fsub_rn(s0, sc_prev));
-              const uint32_t l1 = __float_as_uint(__fsub_rn(s1, s0));
-              v[2 * q] = __funnelshift_l(l0, l0, 1);
-              v[2 * q + 1] = __funnelshift_l(l1, l1, 1);
-              sc_prev = s1;
-            }
-            if (__any_sync(kFull, resmax > eb)) {      // R2's correction somewhere in the warp: redo exactly
-              uint32_t prev = kRoundMagicBits;
+          for (int q = 0; q < 8; ++q) {
+            if ((2 * q) % SL == 0) sc_prev = 0.0f;
+            const uint64_t rs = quantize_scaled2(x[2 * q], x[2 * q + 1], two_eb, recip, vmax, resmax);
+            float s0, s1;
+            asm("mov.b64 {%0, %1}, %2;" : "=f"(s0), "=f"(s1) : "l"(rs));
+            // l = r_j - r_{j-1}, exact on the subnormal grid: bits sign | |l|
+            const uint32_t l0 = __float_as_uint(__fsub_rn(s0, sc_prev));
+            const uint32_t l1 = __float_as_uint(__fsub_rn(s1, s0));
+            v[2 * q] = __funnelshift_l(l0, l0, 1);
+            v[2 * q + 1] = __funnelshift_l(l1, l1, 1);
+            sc_prev = s1;
+          }
+          if (__any_sync(kFull, resmax > eb)) {        // R2's correction somewhere in the warp: redo exactly
+            uint32_t prev = kRoundMagicBits;
 #pragma unroll
-              for (int j = 0; j < SL; ++j) {
-                const uint32_t r = quantize_exact(x[j], eb, two_eb, recip, vmax);
-                const int l = int(r - prev);
-                prev = r;
-                v[j] = (uint32_t(l < 0 ? -l : l) << 1) | (uint32_t(l) >> 31);
-              }
+            for (int j = 0; j < 16; ++j) {
+              if (j % SL == 0) prev = kRoundMagicBits;
+              const uint32_t r = quantize_exact(x[j], eb, two_eb, recip, vmax);
+              const int l = int(r - prev);
+              prev = r;
+              v[j] = (uint32_t(l < 0 ? -l : l) << 1) | (uint32_t(l) >> 31);
             }
+          }
+          uint32_t planes[kBL], c[kBL], ct = 0, pmax = 0;
+#pragma unroll
+          for (int bb = 0; bb < kBL; ++bb) {
             uint32_t o = 0;
 #pragma unroll
-            for (int j = 0; j < SL; ++j) o |= v[j];
-            const uint32_t planes = bitlen(o);
-            fcnt[blk] = uint8_t(planes);               // sync: acq_rel count, then mbarrier staged[m]
-            wmax = max(wmax, planes);
-            const uint32_t c = planes * uint32_t(SL / 8);
-            uint32_t incl = c;
+            for (int j = 0; j < SL; ++j) o |= v[bb * SL + j];
+            planes[bb] = bitlen(o);
+            c[bb] = planes[bb] * uint32_t(SL / 8);
+            ct += c[bb];
+            pmax = max(pmax, planes[bb]);
+          }
+          if constexpr (kBL == 2) *reinterpret_cast<uint16_t*>(fcnt + 2 * lane) = uint16_t(planes[0] | (planes[1] << 8));  // sync: acq_rel count, then mbarrier staged[m]
+          else fcnt[lane] = uint8_t(planes[0]);        // sync: acq_rel count, then mbarrier staged[m]
+          wmax = max(wmax, pmax);
+          uint32_t incl = ct;
 #pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-              const uint32_t y = __shfl_up_sync(kFull, incl, d);
-              if (lane >= d) incl += y;
-            }
-            const uint32_t total = __shfl_sync(kFull, incl, 31);
-            while (cursor + total + 4 > room) {        // the pass's bytes (+ the shared word) must fit
-              room = kRB - (head - ld_volatile_u32(&sm.tail[w]));
-              if (cursor + total + 4 > room) __nanosleep(CUSZP_C_POLL_NS);
-            }
-            // zero the pass's ring words ahead of the OR-ed shared words (all but
-            // a first word shared with the previous pass, whose later bytes are
-            // zero already)
-            {
-              const uint32_t B = head + cursor, E = B + total;
-              for (uint32_t k = ((B + 3) >> 2) + lane; k < ((E + 3) >> 2); k += 32) ring[k & (kRing - 1)] = 0u;  // sync: free ring space (room checked); own warp's words
-              __syncwarp();
-            }
-            const uint32_t X = head + cursor + incl - c;  // ring byte of the block's first byte
-            cursor += total;
+          for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, incl, d);
+            if (lane >= d) incl += y;
+          }
+          const uint32_t total = __shfl_sync(kFull, incl, 31);
+          while (cursor + total + 4 > room) {          // the tile's bytes (+ the shared word) must fit
+            room = kRB - (head - ld_volatile_u32(&sm.tail[w]));
+            if (cursor + total + 4 > room) __nanosleep(CUSZP_C_POLL_NS);
+          }
+          // zero the ring words ahead of the OR-ed shared words (all but a
+          // first word shared with the previous tile, whose later bytes are
+          // zero already)
+          {
+            const uint32_t B = head + cursor, E = B + total;
+            for (uint32_t k = ((B + 3) >> 2) + lane; k < ((E + 3) >> 2); k += 32) ring[k & (kRing - 1)] = 0u;  // sync: free ring space (room checked); own warp's words
+            __syncwarp();
+          }
+          const uint32_t G = (__reduce_max_sync(kFull, pmax) + 7) >> 3;
+          uint32_t X = head + cursor + incl - ct;      // ring byte of the lane's first block
+          cursor += total;
+#pragma unroll
+          for (int bb = 0; bb < kBL; ++bb) {
             const uint32_t sh = 8 * (X & 3u), w0 = X >> 2;
-            const uint32_t nwords = c ? ((X & 3u) + c + 3) >> 2 : 0u;
-            const uint32_t G = (__reduce_max_sync(kFull, planes) + 7) >> 3;
+            const uint32_t nwords = c[bb] ? ((X & 3u) + c[bb] + 3) >> 2 : 0u;
+            X += c[bb];
             // word j of the block (aligned ring word w0 + j): words 1 .. nwords-2
             // lie inside the block and are stored; word 0 and word nwords-1 may
             // share bytes with the neighbouring blocks and are OR-ed in at the end
@@ -794,7 +805,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             for (int g = 0; g < 4; ++g) {
               if (uint32_t(g) < G) {
                 uint32_t sq[kW];
-                block_seq8<SL>(v, uint32_t(g), sq);
+                block_seq8<SL>(v + bb * SL, uint32_t(g), sq);
 #pragma unroll
                 for (int i = 0; i < kW; ++i) {
                   const uint32_t word = __funnelshift_l(prev, sq[i], sh);
