@@ -24,6 +24,11 @@
 //               their global offsets and release ring space in tile order.
 //               Up to kMeta tiles wait for their prefix while the compute
 //               warps keep going, so the look-back latency stays hidden.
+// Block lengths L = 64 / 128 (M = L/32 sub-blocks per block) reuse the L = 32
+// encode; L = 8 / 16 (SL) encode one block per LANE (16 consecutive floats
+// per lane: 2 blocks of 8 or 1 of 16) with in-register 8x8 bit transposes
+// and byte-granular rings, look-back and copy-out.  D = 2 / 3
+// (multi-dimensional Lorenzo, R18): the producer gathers blocks with cp.async.
 #include "internal.cuh"
 
 namespace cuszp {

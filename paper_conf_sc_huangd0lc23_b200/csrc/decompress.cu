@@ -19,6 +19,9 @@
 //     a11 inverse Lorenzo: 4 consecutive elements per lane, 8 lanes per block,
 //         3 local adds + a 3-step segmented shuffle scan,
 //     a12 dequantise d' = (float) r * 2eb (R13), 128-bit stores.
+// L = 8 / 16 (SL): look-back units are bytes; the scanner sums the block
+// bytes of whole warp slices, the loader also stages the tile's F bytes, and
+// each compute lane decodes one block in registers.
 // Every read is bounded by in_bytes (corrupt input -> async ECORRUPT).
 #include <type_traits>
 
