@@ -112,6 +112,10 @@ def main():
     ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
     for it in range(4):
         traced = it == 3
+        if traced:
+            trace.zero_()
+            trace[nt * 8: nt * 8 + 4] = (1 << 62)          # atomicMin slots
+            trace[nt * 8 + 2] = 0
         h.cuszp_debug_set_trace(trace.data_ptr() if traced else None)
         flush.zero_()
         h.cuszp_range(x.data_ptr(), n, mm.data_ptr(), ws.data_ptr(), ws.numel(), sp)
@@ -122,6 +126,11 @@ def main():
         if traced:
             torch.cuda.synchronize()
             trc = trace[: nt * 8].view(nt, 8).cpu().numpy().astype(np.int64)
+            kk = trace[nt * 8: nt * 8 + 4].cpu().numpy().astype(np.int64)
+            t0c = trc[:, 0].min()
+            print(f"compress kernel points rel. first ticket (us): first entry {(kk[0] - t0c) / 1e3:.2f}, "
+                  f"past pdl_wait {(kk[1] - t0c) / 1e3:.2f}, past prologue {(kk[3] - t0c) / 1e3:.2f}, "
+                  f"last prefix {(trc[:, 4].max() - t0c) / 1e3:.2f}, finish {(kk[2] - t0c) / 1e3:.2f}")
             trace.zero_()
             trace[: nt * 8].view(nt, 8)[:, 4] = (1 << 62)
         if a.L != 32:
