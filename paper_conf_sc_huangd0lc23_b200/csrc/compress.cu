@@ -354,7 +354,16 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
   CompressSmem<kWB>& sm = *reinterpret_cast<CompressSmem<kWB>*>(smem_raw);
   const int lane = threadIdx.x & 31;
   const int warp = __shfl_sync(0xffffffffu, int(threadIdx.x >> 5), 0);   // provably warp-uniform (no divergence checks before warp-sync ops)
+#ifdef CUSZP_TRACE
+  // kernel-level points after the per-tile area: [0] first CTA entry, [1] first
+  // CTA past pdl_wait, [2] last CTA done (finish), [3] first CTA past the prologue
+  uint64_t* tr_k = a.trace ? a.trace + 8ull * a.num_tiles : nullptr;
+  if (tr_k && threadIdx.x == 0) atomicMin(reinterpret_cast<unsigned long long*>(tr_k), global_ns());
+#endif
   pdl_wait();                                     // range kernel / previous call complete
+#ifdef CUSZP_TRACE
+  if (tr_k && threadIdx.x == 0) atomicMin(reinterpret_cast<unsigned long long*>(tr_k + 1), global_ns());
+#endif
   pdl_launch_dependents();
   const uint32_t epoch = running_epoch(a.ws);
 
@@ -392,6 +401,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
     fence_mbar_init();
   }
   __syncthreads();
+#ifdef CUSZP_TRACE
+  if (tr_k && threadIdx.x == 0) atomicMin(reinterpret_cast<unsigned long long*>(tr_k + 3), global_ns());
+#endif
 
   if (eb_ok) {
     if (D > 1 && warp == 0) {
@@ -1050,6 +1062,9 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
       if (a.out_bytes) *a.out_bytes = (a.n == 0) ? uint64_t(kHdr) : p0 + payload_bytes;
     }
     finish_call(a.ws, a.status, a.status_cap, epoch, final_status);
+#ifdef CUSZP_TRACE
+    if (tr_k && threadIdx.x == 0) tr_k[2] = global_ns();
+#endif
   }
 }
 
