@@ -131,6 +131,17 @@ def main():
             print(f"compress kernel points rel. first ticket (us): first entry {(kk[0] - t0c) / 1e3:.2f}, "
                   f"past pdl_wait {(kk[1] - t0c) / 1e3:.2f}, past prologue {(kk[3] - t0c) / 1e3:.2f}, "
                   f"last prefix {(trc[:, 4].max() - t0c) / 1e3:.2f}, finish {(kk[2] - t0c) / 1e3:.2f}")
+            rec = trace[nt * 8: nt * 16].view(nt, 8).cpu().numpy().astype(np.int64)[:, 4:]
+            if rec[1:, 0].any():
+                # in-place kernels: recycler / writer points (slots 4-7 of region 2)
+                sel = slice(1, None)
+                agg_t = trc[sel, 2]
+                print("in-place compress, per tile (us):")
+                print(f"  aggregate -> recycler picks up  {pct((rec[sel, 0] - agg_t) / 1e3)}")
+                print(f"  picked up -> room/slot ok      {pct((rec[sel, 1] - rec[sel, 0]) / 1e3)}")
+                print(f"  room ok -> parked (stage free) {pct((rec[sel, 2] - rec[sel, 1]) / 1e3)}")
+                print(f"  prefix -> released             {pct((rec[sel, 3] - trc[sel, 4]) / 1e3)}")
+                print(f"  parked -> released             {pct((rec[sel, 3] - rec[sel, 2]) / 1e3)}")
             trace.zero_()
             trace[: nt * 8].view(nt, 8)[:, 4] = (1 << 62)
         if a.L != 32:
