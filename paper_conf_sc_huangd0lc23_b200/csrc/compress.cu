@@ -945,6 +945,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           wmax = max(wmax, span);
           const uint32_t wb = pack4(wq[0], wq[1], wq[2], wq[3]);
           const uint32_t base = head + cursor;
+#ifndef CUSZP_DIAG_NOXPOSE   // (diagnostics only: no transposes / ring stores, garbage output)
           if (M > 1) {
             // word k of sub-block q -> block payload position M k + q % M
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 100)
@@ -990,6 +991,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
               o += wq[q];
             }
           }
+#endif
           cursor += (wb * 0x01010101u) >> 24;                          // sum of the 4 counts
 #if CUSZP_C_GUNROLL >= 4
           wbs[g] = wb;

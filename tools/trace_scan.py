@@ -64,6 +64,8 @@ def report(name, tr, total_ns):
     print(f"  look-back duration      (us) {pct(pfx - lb0)}")
     print(f"  ticket -> prefix        (us) {pct(pfx - ticket)}")
     print(f"  windows {pct(tr[:, 5])}   spins {pct(tr[:, 6])}")
+    print(f"  windows mean {tr[:, 5].mean():.2f} max {tr[:, 5].max()}   spins mean {tr[:, 6].mean():.2f} max {tr[:, 6].max()}"
+          f"  (sum {tr[:, 6].sum()})")
     # lag: at each prefix time, how many tiles with smaller index had no aggregate yet
     order = np.argsort(tr[:, 2])
     print(f"  aggregate order vs ticket order: mean |rank diff| = {np.abs(np.argsort(order) - np.arange(len(order))).mean():.1f}")
