@@ -66,6 +66,7 @@ def parse_args():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-secondary", action="store_true", help="skip the c1/c2/c4/c5 secondary keys")
     p.add_argument("--no-variants", action="store_true", help="skip the block-length / predictor variants")
+    p.add_argument("--no-datasets", action="store_true", help="skip the six-dataset table")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     return p.parse_args()
@@ -650,6 +651,47 @@ def variants(r: Runner, peak: float, steps: int) -> dict:
     return out
 
 
+PAPER_DATASETS = {
+    "compress_gbs": {"CESM-ATM": 41.77, "QMCPack": 140.44},
+    "decompress_gbs": {"CESM-ATM": 49.91, "NYX": 190.11},
+    "source": "PAPER.md P:963-966 (A100, end-to-end, real data, mean over REL 1E-1..1E-4; the other "
+              "per-dataset bars of Fig 13 are not legible in the text)"}
+
+
+def datasets_table(peak: float, steps: int, dev) -> dict:
+    """The paper's six datasets (Table 2, one field shape each; synth.DATASETS)
+    at REL 1e-2 / 1e-3 / 1e-4: GB/s of fp32 input for REL compression (range +
+    compress kernel, the paper's end-to-end compression), decompression, the
+    round trip, CR per bound, and each kernel's fraction of the HBM peak;
+    L2 flushed before every round trip, every stream's status checked."""
+    import synth
+
+    r = Runner(dev, max(280_953_867, 512 ** 3))
+    out = {"rel": synth.DATASET_RELS, "unit": "GB/s of fp32 input", "steps": steps}
+    for name, spec in synth.DATASETS.items():
+        xs = {f: synth.dataset_field(name, f, dev) for f in spec["fields"]}
+        jobs = [(f"{f}@{rel:g}", xs[f], xs[f].numel(), rel) for f in spec["fields"] for rel in synth.DATASET_RELS]
+        acc, sizes, _, _ = r.measure(jobs, steps, 3)
+        d = summarise(jobs, acc, sizes, steps, 1, peak)
+        cr = {}
+        for rel in synth.DATASET_RELS:
+            labs = [f"{f}@{rel:g}" for f in spec["fields"]]
+            n_in = sum(4 * xs[f].numel() for f in spec["fields"])
+            cr[f"{rel:g}"] = round(n_in / sum(sizes[lab] for lab in labs), 3)     # aggregate over the fields
+        out[name] = {"dims_per_field": spec["dims"], "fields": spec["fields"],
+                     "n_per_field": [xs[f].numel() for f in spec["fields"]],
+                     "compress_gbs": round(d["compress_gbs"], 1), "decompress_gbs": round(d["decompress_gbs"], 1),
+                     "round_trip_gbs": round(d["round_trip_gbs"], 1), "cr": cr,
+                     "rel_compress_frac_of_peak": round(d["rel_compress_frac_of_peak"], 4),
+                     "frac_of_peak": {k: round(v["frac_of_peak"], 4) for k, v in d["kernels"].items()}}
+        del xs, jobs
+        torch.cuda.empty_cache()
+    out["paper_context"] = PAPER_DATASETS
+    del r
+    torch.cuda.empty_cache()
+    return out
+
+
 def verify(r: Runner, jobs) -> dict:
     """Every job's round trip checked on the device with the fused quality
     kernel (cuszp_quality, untimed): the bound of DESIGN sec 5 and PSNR."""
@@ -756,6 +798,8 @@ def run_ours(args, rank, world, dev):
     if world == 1 and not args.no_variants:
         line["block_len_variants"] = variants(Runner(dev, 25_000_000), peak, 5)
         torch.cuda.empty_cache()
+    if world == 1 and not args.no_datasets:
+        line["datasets"] = datasets_table(peak, 3, dev)
     return line
 
 

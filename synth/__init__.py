@@ -11,6 +11,9 @@ takes a ``device`` so large fields are built directly in HBM.
 """
 from .fields import (  # noqa: F401
     CONFIGS,
+    DATASET_RELS,
+    DATASETS,
+    dataset_field,
     field_for_config,
     hacc_like,
     hurricane_like,

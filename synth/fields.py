@@ -167,16 +167,23 @@ def _ricker(t: torch.Tensor) -> torch.Tensor:
 
 
 def rtm_like(nsnap: int = 36, shape=(449, 449, 235), seed: int = 7, device="cpu",
-             out: torch.Tensor | None = None) -> torch.Tensor:
+             out: torch.Tensor | None = None, snaps=None) -> torch.Tensor:
     """Seismic wavefield snapshots (1 per 100 of 3600 steps):
     a Ricker wavefront expanding from a near-surface source with 1/r
-    spreading and reflections from 3 layers; EXACTLY 0 ahead of every front,
-    so early snapshots are sparse and late ones dense (Fig 22).
-    Shape (nsnap, X, Y, Z) flattened C-order; the set is one 1D array."""
+    spreading and reflections from 3 layers; EXACTLY 0 ahead of every front
+    (and behind it once the pulse has passed: the Ricker tail underflows), so
+    the non-zero fraction grows while the front crosses the box (0.3 % at
+    t0, 40 % at t14: "sparse early", Fig 22) and falls again
+    as it leaves (all zero from ~t25).  Set CR at 1e-3: 44.3 (paper's RTM
+    average 42.40, Table 3).
+    Shape (nsnap, X, Y, Z) flattened C-order; the set is one 1D array.
+    ``snaps``: only these snapshot indices (each identical to its slice of the
+    whole set), concatenated in the given order."""
     X, Y, Z = shape
     per = X * Y * Z
+    snaps = list(range(nsnap)) if snaps is None else list(snaps)
     if out is None:
-        out = torch.empty(nsnap * per, dtype=torch.float32, device=device)
+        out = torch.empty(len(snaps) * per, dtype=torch.float32, device=device)
     g = _gen(seed, device)
     src = torch.tensor([0.5 * X, 0.5 * Y, 12.0], device=device)
     src = src + torch.rand(3, generator=g, device=device) * 4.0
@@ -188,7 +195,7 @@ def rtm_like(nsnap: int = 36, shape=(449, 449, 235), seed: int = 7, device="cpu"
     zs = torch.arange(Z, device=device, dtype=torch.float32).view(1, 1, Z)
     dxy = (xs - src[0]) ** 2 + (ys - src[1]) ** 2
     width = 6.0
-    for s in range(nsnap):
+    for k, s in enumerate(snaps):
         R = (s + 1) / nsnap * 1.05 * diag
         snap = torch.zeros((X, Y, Z), dtype=torch.float32, device=device)
         r = torch.sqrt(dxy + (zs - src[2]) ** 2) + 1.0
@@ -201,7 +208,7 @@ def rtm_like(nsnap: int = 36, shape=(449, 449, 235), seed: int = 7, device="cpu"
                 m = (ri <= R + 2.5 * width) & (zs <= zl)
                 snap += torch.where(m, c * _ricker((ri - R) / width) * (200.0 / ri), torch.zeros((), device=device))
                 del ri, m
-        out[s * per:(s + 1) * per] = snap.reshape(-1)
+        out[k * per:(k + 1) * per] = snap.reshape(-1)
         del snap, r, arg
     return out
 
@@ -240,6 +247,38 @@ CONFIGS = {
     "c4_nyx": dict(shape=(512, 512, 512), rel=[1e-4], seed=6),
     "c5_rtm": dict(nsnap=36, shape=(449, 449, 235), rel=[1e-3], seed=7),
 }
+
+
+# the paper's six datasets (Table 2), one entry per FIELD shape
+# (dims per field), REL 1e-2 / 1e-3 / 1e-4 (the paper averages 1e-1 .. 1e-4,
+# P:945-948): the bench's six-dataset throughput table
+DATASETS = {
+    "Hurricane": dict(fields=["U", "QCLOUD", "TC"], dims="100x500x500"),
+    "NYX": dict(fields=["temperature"], dims="512x512x512"),
+    "QMCPack": dict(fields=["orbitals"], dims="288x115x69x69"),
+    "RTM": dict(fields=["t04", "t09", "t14"], dims="449x449x235 (snapshots 4, 9, 14 of 36: the growing front)"),
+    "HACC": dict(fields=["x"], dims="280,953,867"),
+    "CESM-ATM": dict(fields=["T"], dims="1800x3600"),
+}
+DATASET_RELS = [1e-2, 1e-3, 1e-4]
+
+
+def dataset_field(name: str, field: str, device="cpu") -> torch.Tensor:
+    """One field of a DATASETS entry as a flat fp32 tensor."""
+    if name == "Hurricane":
+        return field_for_config("c2_hurricane", device=device, field=field)
+    if name == "NYX":
+        return field_for_config("c4_nyx", device=device)
+    if name == "QMCPack":
+        return qmcpack_like(device=device)
+    if name == "RTM":
+        c = CONFIGS["c5_rtm"]
+        return rtm_like(c["nsnap"], c["shape"], c["seed"], device, snaps=[int(field[1:])])
+    if name == "HACC":
+        return field_for_config("c3_hacc", device=device)
+    if name == "CESM-ATM":
+        return cesm_like(device=device).reshape(-1)
+    raise KeyError(name)
 
 
 def _scaled(shape, scale: float):

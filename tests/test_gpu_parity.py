@@ -280,6 +280,32 @@ def test_full_size_bytes(name):
 
 
 @pytest.mark.slow
+@pytest.mark.parametrize("name", list(synth.DATASETS))
+def test_full_size_datasets(name):
+    """The bench's six-dataset table (synth.DATASETS: the paper's Table 2 field
+    shapes) at every bound it reports, REL 1e-2 / 1e-3 / 1e-4:
+    every field's whole stream and whole reconstruction against the oracle,
+    in the launch configuration bench.py times."""
+    for f in synth.DATASETS[name]["fields"]:
+        x = synth.dataset_field(name, f, device=DEV)
+        x_np = x.cpu().numpy()
+        for rel in synth.DATASET_RELS:
+            st, s_o = oracle.compress(x_np, rel, oracle.REL)
+            assert st == oracle.OK, (name, f, rel, st)
+            out, nb = cz.compress(x, rel, "rel")
+            torch.cuda.synchronize()
+            assert int(nb.item()) == s_o.size, (name, f, rel)
+            assert _equal_chunked(out[: s_o.size], s_o), (name, f, rel)
+            y = cz.decompress(out, x.numel(), in_bytes=int(nb.item()))
+            st, y_o = oracle.decompress(s_o, x_np.size)
+            assert st == oracle.OK
+            assert _equal_chunked(y, y_o), (name, f, rel)
+            del out, y, y_o, s_o
+        del x, x_np
+        torch.cuda.empty_cache()
+
+
+@pytest.mark.slow
 def test_full_size_rtm_bit_exact():
     """The 6.82 GB RTM-shaped set (BASELINE configs[4], 1,705,544,460 fp32),
     every byte and every float:
