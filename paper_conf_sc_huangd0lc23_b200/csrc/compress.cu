@@ -636,7 +636,11 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         } else {
         uint32_t* dst_t = payload + excl + lane;
 #pragma unroll 1
+#ifdef CUSZP_DIAG_NOCOPY
+        for (int w = 0; w < 0; ++w) {   // diagnostics only: no copy-out (garbage payload)
+#else
         for (int w = 0; w < kCW; ++w) {
+#endif
           const uint32_t c = __shfl_sync(kFull, cnt, w);
           const uint32_t h = __shfl_sync(kFull, hd, w);
           const uint32_t off = __shfl_sync(kFull, incl - cnt, w);
