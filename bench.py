@@ -425,10 +425,14 @@ def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int)
     # out), each job's decompression event-ordered after its compression, so
     # the two directions of the link carry balanced traffic at all times.
     n_sets = int(os.environ.get("CUSZP_E2E_LANES", "2"))
+    # host stream buffers per set: with 2, a compression only waits for the
+    # decompression that read the same buffer two rounds ago
+    n_hbuf = int(os.environ.get("CUSZP_E2E_HBUF", "1"))
     sets = []
     for _ in range(n_sets):
         sets.append(dict(cs=torch.cuda.Stream(dev), ds=torch.cuda.Stream(dev),
-                         h_out=torch.zeros(cap, dtype=torch.uint8).pin_memory(),
+                         h_outs=[torch.zeros(cap, dtype=torch.uint8).pin_memory() for _ in range(n_hbuf)],
+                         dec_dones=[torch.cuda.Event() for _ in range(n_hbuf)], hb_used=[False] * n_hbuf, use=0,
                          h_len=torch.zeros(1, dtype=torch.int64).pin_memory(),
                          h_y=torch.empty(nmax, dtype=torch.float32).pin_memory(),
                          d_in=torch.empty(nmax, dtype=torch.float32, device=dev),
@@ -449,16 +453,19 @@ def e2e_measure(cz, dev, jobs_host, steps: int, world: int, cap: int, nmax: int)
             st = sets[k % n_sets]
             k += 1
             n = h_in.numel()
-            if st["used"]:
-                st["cs"].wait_event(st["dec_done"])          # h_out is free once the last decompression read it
+            b = st["use"] % n_hbuf
+            st["use"] += 1
+            st["h_out"] = st["h_outs"][b]
+            if st["hb_used"][b]:
+                st["cs"].wait_event(st["dec_dones"][b])      # h_out is free once the decompression that read it is done
             cz.compress_host_async(h_in, rel, "rel", st["h_out"], st["h_len"], st["d_in"][:n], st["d_out"],
                                    st["wsc"], stream=st["cs"])
             st["comp_done"].record(st["cs"])
             st["ds"].wait_event(st["comp_done"])
             cz.decompress_host_async(st["h_out"], st["h_y"][:n], st["d_sin"], st["d_y"][:n], st["wsd"],
                                      stream=st["ds"])
-            st["dec_done"].record(st["ds"])
-            st["used"] = True
+            st["dec_dones"][b].record(st["ds"])
+            st["hb_used"][b] = True
             if i == 0:      # warm-up pass: record the stream lengths (bytes counted per step)
                 st["ds"].synchronize()
                 lens[lab] = int(st["h_len"].item())
