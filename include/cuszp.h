@@ -260,6 +260,26 @@ size_t cuszp_quality_workspace_bytes(void);
 int cuszp_quality(const float* d_x, const float* d_y, size_t n, double bound,
                   cuszp_quality_stats* d_q, void* d_ws, size_t ws_bytes, void* stream);
 
+/* ---- sharded container, one-sided gather ----------
+ * Container v2: u64 words magic "CSZPCONT", version 2,
+ * P, n_total, n_p[P], bytes_p[P], offset_p[P] (offsets of the 16-byte
+ * aligned shards, relative to the header's end), the header padded to 16
+ * bytes.  cuszp_container_put copies shard p (d_shard, this rank's stream,
+ * 16-byte aligned) into the container at d_container (any device address
+ * the calling GPU can write: its own memory or a peer GPU's, mapped by CUDA
+ * IPC / UVA; 16-byte aligned) at the offset d_header (the container header
+ * words, device memory, 8-byte aligned) gives it -- read ON THE DEVICE, so a
+ * gather needs no host round trip -- followed by zeros up to align16(bytes_p)
+ * (so d_container needs room for the padded shard); with write_header != 0
+ * it also writes the header words and their zero padding.  The caller orders the puts of
+ * all ranks before the container is read (e.g. an NCCL all-reduce after the
+ * put on every rank's stream).  Sync errors: EINVAL (NULL pointers, P = 0,
+ * p >= P, misalignment), ECUDA; the copy itself has no data-dependent
+ * errors (bytes_p and offset_p are trusted: they come from the all-gather
+ * of the compressed sizes). */
+int cuszp_container_put(const void* d_shard, const void* d_header, unsigned P, unsigned p, void* d_container,
+                        int write_header, void* stream);
+
 /* Human-readable status name. */
 const char* cuszp_status_string(int status);
 

@@ -27,7 +27,7 @@ SYMBOLS = (
     "cuszp_compress_L", "cuszp_compress_minmax_L", "cuszp_decompress_L", "cuszp_max_compressed_bytes_L",
     "cuszp_compress_ex", "cuszp_decompress_ex",
     "cuszp_num_blocks_md", "cuszp_max_compressed_bytes_md", "cuszp_workspace_bytes_md", "cuszp_compress_md",
-    "cuszp_decompress_md",
+    "cuszp_decompress_md", "cuszp_container_put",
 )
 
 _lock = threading.Lock()
@@ -93,6 +93,8 @@ def _declare(h):
     h.cuszp_compress_md.restype = i32
     h.cuszp_decompress_md.argtypes = [vp, sz, vp, sz, sz, sz, i32, vp, sz, vp]
     h.cuszp_decompress_md.restype = i32
+    h.cuszp_container_put.argtypes = [vp, vp, C.c_uint, C.c_uint, vp, i32, vp]
+    h.cuszp_container_put.restype = i32
     h.cuszp_version.argtypes = []
     h.cuszp_version.restype = i32
 

@@ -547,6 +547,16 @@ int cuszp_decompress_host_async(const void* h_in, size_t in_capacity, float* h_o
   return CUSZP_OK;
 }
 
+int cuszp_container_put(const void* d_shard, const void* d_header, unsigned P, unsigned p, void* d_container,
+                        int write_header, void* stream) {
+  if (d_shard == nullptr || d_header == nullptr || d_container == nullptr || P == 0 || p >= P) return CUSZP_EINVAL;
+  if (misaligned(d_shard, 16) || misaligned(d_container, 16) || misaligned(d_header, 8)) return CUSZP_EINVAL;
+  DeviceInfo di;
+  if (device_info(&di) != CUSZP_OK) return CUSZP_ECUDA;
+  return launch_container_put(d_shard, d_header, P, p, d_container, write_header, di.sms,
+                              static_cast<cudaStream_t>(stream));
+}
+
 const char* cuszp_status_string(int status) {
   switch (status) {
     case CUSZP_OK: return "CUSZP_OK";

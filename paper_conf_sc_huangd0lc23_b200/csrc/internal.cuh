@@ -503,6 +503,8 @@ __global__ void range_kernel(RangeArgs a);
 int launch_copy_len(void* dst, const void* src, const unsigned long long* d_len, uint64_t cap,
                     unsigned long long* len_out, int sms, cudaStream_t s);
 int launch_stream_len(const void* h_stream_dev, uint64_t n, unsigned long long* d_len, cudaStream_t s);
+int launch_container_put(const void* shard, const void* hdr, uint32_t P, uint32_t p, void* cont, int write_header,
+                         int sms, cudaStream_t s);
 size_t compress_smem_bytes();
 int compress_threads();
 size_t decompress_smem_bytes();

@@ -21,6 +21,9 @@ decompression:
     buffer (header words + every shard at a 16-byte aligned offset) on one
     rank (NCCL point-to-point receives straight into the slices) or on every
     rank (one NCCL broadcast per shard into its slice);
+    ``gather_container_p2p``: the same container on one rank with no host
+    read of the sizes -- every rank's copy kernel writes its shard into the
+    root's (IPC-mapped) buffer at the offset the device-side header gives;
  4. ``decompress_container``: decompresses all shards of a container on one
     GPU (one launch per shard, each writing its slab of the output), and
     ``decompress_sharded`` + ``allgather_slabs`` decompress a container
@@ -242,6 +245,69 @@ def gather_container(res: ShardResult, group=None, dst: int | None = None) -> to
                 dist.recv(tmp, src=src, group=group)
                 views[p].copy_(tmp)
     return buf
+
+
+def container_capacity(shard_n: list[int]) -> int:
+    """Bytes that hold a container of these shards whatever their sizes: the
+    header plus every shard's align16(cuszp_max_compressed_bytes(n_p))."""
+    import paper_conf_sc_huangd0lc23_b200 as cz
+
+    return container_header_bytes(len(shard_n)) + sum((cz.max_compressed_bytes(n) + 15) // 16 * 16 for n in shard_n)
+
+
+_peer_cache: dict = {}
+
+
+def _peer_view(buf: torch.Tensor | None, dst: int, group, cache_key=None) -> torch.Tensor:
+    """Every rank gets a device tensor aliasing rank dst's ``buf`` (CUDA IPC:
+    the handle travels as a small host object; a rank on another GPU then
+    writes it over NVLink / UVA).  With a cache_key the mapping is made once
+    and reused by every later call with that key -- ALL ranks must pass the
+    same keys, and dst the same buffer for a key."""
+    from torch.multiprocessing.reductions import reduce_tensor
+
+    if cache_key is not None and cache_key in _peer_cache:
+        return _peer_cache[cache_key][0]
+    rank = dist.get_rank(group)
+    obj = [reduce_tensor(buf) if rank == dst else None]
+    dist.broadcast_object_list(obj, src=dist.get_global_rank(group, dst) if group is not None else dst, group=group)
+    view = buf if rank == dst else obj[0][0](*obj[0][1])
+    if cache_key is not None:
+        _peer_cache[cache_key] = (view, obj[0])
+    return view
+
+
+def gather_container_p2p(res: ShardResult, shard_n: list[int], group=None, dst: int = 0,
+                         buf: torch.Tensor | None = None, cache_key=None) -> torch.Tensor | None:
+    """One-sided gather of the container on rank ``dst`` with no host read
+    of the sizes: every rank's copy kernel (cuszp_container_put) writes its
+    shard straight into dst's buffer -- mapped by CUDA IPC, so over NVLink
+    when dst is another GPU -- at the offset the DEVICE-side header gives it,
+    and rank dst writes the header.  An all-reduce of one word after the put
+    (stream-ordered under NCCL) orders every rank's put before dst reads the
+    container.  ``buf`` (dst only): a container_capacity(shard_n)-byte device
+    buffer; with ``cache_key`` (same on every rank) its IPC mapping is made
+    once and reused.  Returns the buffer on dst (the container occupies its
+    first container_total_bytes(header) bytes), None elsewhere."""
+    import paper_conf_sc_huangd0lc23_b200 as cz
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    dev = res.stream.device
+    if rank == dst and buf is None:
+        buf = torch.empty(container_capacity(shard_n), dtype=torch.uint8, device=dev)
+    view = _peer_view(buf, dst, group, cache_key) if world > 1 else buf
+    s = torch.cuda.current_stream(dev)
+    cz.check(cz.lib().cuszp_container_put(res.stream.data_ptr(), res.header.data_ptr(), world, rank, view.data_ptr(),
+                                          1 if rank == dst else 0, s.cuda_stream), "container_put")
+    if world > 1:
+        if _nccl(group):
+            tok = torch.zeros(1, dtype=torch.int32, device=dev)
+            dist.all_reduce(tok, group=group)                # after every put on every rank's stream
+        else:
+            torch.cuda.synchronize(dev)                      # gloo (tests): host-ordered
+            dist.barrier(group=group)
+    return buf if rank == dst else None
 
 
 def container_shards(buf: torch.Tensor) -> tuple[dict, list[torch.Tensor]]:

@@ -32,6 +32,9 @@ def main():
     res = czd.compress_sharded(x[s0:s1].contiguous(), 1e-3, shard_n)
     buf = czd.gather_container(res)
     root = czd.gather_container(res, dst=0)
+    root_p2p = czd.gather_container_p2p(res, shard_n, dst=0)          # one-sided, IPC-mapped root buffer
+    root_p2p2 = czd.gather_container_p2p(res, shard_n, dst=world - 1, cache_key="last")   # another root, cached mapping
+    root_p2p3 = czd.gather_container_p2p(res, shard_n, dst=world - 1, buf=root_p2p2, cache_key="last")
     local = czd.decompress_sharded(buf)
     full = czd.allgather_slabs(local, shard_n)
     x_np = x.cpu().numpy()
@@ -43,6 +46,9 @@ def main():
     ok &= np.array_equal(full.cpu().numpy().view(np.uint32), y_o.view(np.uint32))
     if rank == 0:
         ok &= torch.equal(buf, root)
+        ok &= torch.equal(root_p2p[: buf.numel()], buf)
+    if rank == world - 1:
+        ok &= torch.equal(root_p2p2[: buf.numel()], buf) and torch.equal(root_p2p3[: buf.numel()], buf)
     flag = torch.tensor([1 if ok else 0], device=dev if not share else "cpu")
     dist.all_reduce(flag, op=dist.ReduceOp.MIN)
     if rank == 0:
