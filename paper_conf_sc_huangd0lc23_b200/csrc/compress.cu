@@ -65,6 +65,9 @@ namespace {
 #ifndef CUSZP_C_L2_AHEAD
 #define CUSZP_C_L2_AHEAD 1       // > 0: prefetch the input tile this many grids ahead into L2
 #endif
+#ifndef CUSZP_C_COPY_UNROLLED
+#define CUSZP_C_COPY_UNROLLED 1  // copy-out of a ring segment in unrolled groups of 4 chunks (0: the round-2 loop)
+#endif
 #ifndef CUSZP_C_FULL_POLL_NS
 #define CUSZP_C_FULL_POLL_NS 0   // > 0: compute warps poll their input stage with test + nanosleep
 #endif
@@ -645,6 +648,32 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           const uint32_t h = __shfl_sync(kFull, hd, w);
           const uint32_t off = __shfl_sync(kFull, incl - cnt, w);
           const uint32_t first = min(c, kRing - h);               // words before the wrap
+#if CUSZP_C_COPY_UNROLLED
+          // a segment is <= 16 x 32 words: groups of 4 chunks, fully unrolled
+          // (immediate offsets, a lane test per chunk, one warp-uniform exit
+          // test per group; no pointer updates, no remainder loop)
+          {
+            uint32_t* dst = dst_t + off;
+            const uint32_t* src = sm.ring[w] + h + lane;
+#pragma unroll
+            for (int i = 0; i < kCBPW; i += 4) {
+              if (32u * i >= first) break;
+#pragma unroll
+              for (int j = i; j < i + 4; ++j)
+                if (lane + 32u * j < first) dst[32 * j] = src[32 * j];  // sync: ring written before staged[m]; reused only after the tail release
+            }
+            dst = dst_t + off + first;
+            src = sm.ring[w] + lane;
+            const uint32_t rest = c - first;
+#pragma unroll
+            for (int i = 0; i < kCBPW; i += 4) {
+              if (32u * i >= rest) break;
+#pragma unroll
+              for (int j = i; j < i + 4; ++j)
+                if (lane + 32u * j < rest) dst[32 * j] = src[32 * j];  // sync: as above
+            }
+          }
+#else
           uint32_t* dst = dst_t + off;
           const uint32_t* src = sm.ring[w] + h + lane;
 #pragma unroll 4
@@ -653,6 +682,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           dst = dst_t + off + first;
 #pragma unroll 2
           for (int k = lane; k < int(c - first); k += 32, src += 32, dst += 32) *dst = *src;  // sync: ring written before staged[m]; reused only after the tail release
+#endif
         }
         }
         // release ring space in CTA tile order
