@@ -241,6 +241,14 @@ __device__ __forceinline__ void stress_delay(uint32_t) {}
 #endif
 
 // ------------------------------------------------------------- warp helpers
+// sum over the warp of values < 2^44 (look-back parts: <= K aggregates /
+// prefixes of <= 40 bits): two 32-bit REDUX.SUMs of the low 24 and the high
+// bits (each sum fits 32 bits) instead of five 64-bit shuffle rounds
+__device__ __forceinline__ uint64_t warp_sum_u44(uint64_t v) {
+  const uint32_t lo = __reduce_add_sync(kFull, uint32_t(v) & 0xFFFFFFu);
+  const uint32_t hi = __reduce_add_sync(kFull, uint32_t(v >> 24));
+  return (uint64_t(hi) << 24) + lo;
+}
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
@@ -289,6 +297,7 @@ __device__ __forceinline__ uint64_t resolve_excl(const uint64_t* status, uint32_
                                                  uint32_t* n_windows = nullptr, uint32_t* n_spins = nullptr) {
   if (t == 0) return 0;
   constexpr int K = CUSZP_LB_K;
+  static_assert(K >= 1 && K <= 16, "a lane's part (<= K values of 40 bits) must stay below 2^44 (warp_sum_u44)");
   uint32_t windows = 0, spins = 0;
   const int lane = threadIdx.x & 31;
   const uint64_t tag = uint64_t(epoch) << kEpochShift;
@@ -323,7 +332,7 @@ __device__ __forceinline__ uint64_t resolve_excl(const uint64_t* status, uint32_
     }
     const uint32_t pmask = __ballot_sync(kFull, has_p);
     const int stop = pmask ? (__ffs(pmask) - 1) : 31;
-    excl += warp_sum_u64(lane <= stop ? part : 0ull);
+    excl += warp_sum_u44(lane <= stop ? part : 0ull);
     if (pmask) break;
     top -= 32 * K;
   }
