@@ -1034,7 +1034,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
 #endif
         }
         __syncwarp();
-        if (lane == 0) {
+        if (elect_one()) {                                 // lane 0 (elect: no warp-aggregated atomic below)
           mbar_arrive(&sm.empty[s]);                       // input stage consumed
           TileMeta<kWB>& md = sm.meta[m];
           // the group word counts go to the writer, which stores the tile's F bytes

@@ -241,6 +241,14 @@ __device__ __forceinline__ void stress_delay(uint32_t) {}
 #endif
 
 // ------------------------------------------------------------- warp helpers
+// one lane of a converged warp (elect.sync): unlike `lane == 0`, ptxas then
+// knows a single lane runs the block and emits its shared-memory atomics
+// as they are (no warp-aggregation sequence around them)
+__device__ __forceinline__ bool elect_one() {
+  uint32_t p;
+  asm volatile("{ .reg .pred P; elect.sync _|P, 0xffffffff; selp.u32 %0, 1, 0, P; }" : "=r"(p));
+  return p != 0;
+}
 // sum over the warp of values < 2^44 (look-back parts: <= K aggregates /
 // prefixes of <= 40 bits): two 32-bit REDUX.SUMs of the low 24 and the high
 // bits (each sum fits 32 bits) instead of five 64-bit shuffle rounds
