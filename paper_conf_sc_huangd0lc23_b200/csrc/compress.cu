@@ -628,12 +628,27 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             if (uint32_t(lane) < tb) g[hb + 4 * nw + lane] = rb[(h + hb + 4 * nw + lane) & kMaskB];  // sync: ring written before staged[m]; reused only after the tail release
             const uint32_t s0 = h + hb, sh = 8 * (s0 & 3u);
             uint32_t* gw = reinterpret_cast<uint32_t*>(g + hb);
+            const uint32_t wm = (s0 >> 2) & (kRing - 1);
+            if (wm + nw + 1 <= kRing) {
+              // no ring wrap (the common case): unrolled groups of 4 chunks of
+              // 32 words with immediate offsets (as the L >= 32 copy-out)
+              const uint32_t* src = rw + wm + lane;
+              uint32_t* dst = gw + lane;
+#pragma unroll
+              for (int i = 0; i < 32; i += 4) {
+                if (32u * i >= nw) break;
+#pragma unroll
+                for (int j = i; j < i + 4; ++j)
+                  if (lane + 32u * j < nw) dst[32 * j] = __funnelshift_r(src[32 * j], src[32 * j + 1], sh);  // sync: ring written before staged[m]; reused only after the tail release
+              }
+            } else {
 #pragma unroll 2
-            for (uint32_t k = lane; k < nw; k += 32) {
-              const uint32_t wi = (s0 >> 2) + k;
-              const uint32_t lo = rw[wi & (kRing - 1)];  // sync: ring written before staged[m]; reused only after the tail release
-              const uint32_t hi = rw[(wi + 1) & (kRing - 1)];  // sync: ring written before staged[m] (bytes past the segment unused)
-              gw[k] = __funnelshift_r(lo, hi, sh);
+              for (uint32_t k = lane; k < nw; k += 32) {
+                const uint32_t wi = (s0 >> 2) + k;
+                const uint32_t lo = rw[wi & (kRing - 1)];  // sync: ring written before staged[m]; reused only after the tail release
+                const uint32_t hi = rw[(wi + 1) & (kRing - 1)];  // sync: ring written before staged[m] (bytes past the segment unused)
+                gw[k] = __funnelshift_r(lo, hi, sh);
+              }
             }
           }
         } else {
