@@ -68,6 +68,9 @@ namespace {
 #ifndef CUSZP_C_COPY_UNROLLED
 #define CUSZP_C_COPY_UNROLLED 1  // copy-out of a ring segment in unrolled groups of 4 chunks (0: the round-2 loop)
 #endif
+#ifndef CUSZP_C_RARE_CALL
+#define CUSZP_C_RARE_CALL 1      // the R2-correction redo of a group as an out-of-line call (L = 32, 1D, order 1)
+#endif
 #ifndef CUSZP_C_FULL_POLL_NS
 #define CUSZP_C_FULL_POLL_NS 0   // > 0: compute warps poll their input stage with test + nanosleep
 #endif
@@ -208,6 +211,16 @@ __device__ __forceinline__ uint32_t lorenzo_pack(uint32_t rb, int lane) {
   const uint32_t a = uint32_t(l < 0 ? -l : l);
   return (a << 1) | (uint32_t(l) >> 31);
 }
+// The R2 correction of one group of 4 blocks (L = 32, 1D, order 1), out of
+// line: the rare redo of the unrolled encode loop (an element within an ulp
+// of a half integer of 2eb) as a call instead of four inlined copies, so the
+// hot loop stays compact.  Returns v of the 4 blocks, their word counts
+// (bytes of wb) and the updated guard maximum; 6 values, returned in
+// registers.
+struct RareOut { uint32_t v0, v1, v2, v3, wb; float vmax; };
+__device__ __noinline__ RareOut rare_group_redo(float x0, float x1, float x2, float x3, float eb, float two_eb,
+                                                float recip, float vmax, int lane);
+
 // same, lane 0 taking `first` (biased) as its predecessor: the last element
 // of the previous 32-element sub-block of an L = 32 M block
 __device__ __forceinline__ uint32_t lorenzo_pack_first(uint32_t rb, int lane, uint32_t first) {
@@ -224,6 +237,18 @@ __device__ __forceinline__ uint32_t bitlen(uint32_t x) {
   uint32_t p;
   asm("bfind.u32 %0, %1;" : "=r"(p) : "r"(x));
   return p + 1u;
+}
+
+__device__ __noinline__ RareOut rare_group_redo(float x0, float x1, float x2, float x3, float eb, float two_eb,
+                                                float recip, float vmax, int lane) {
+  const float xs[4] = {x0, x1, x2, x3};
+  uint32_t v[4], wb = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    v[q] = lorenzo_pack(quantize_exact(xs[q], eb, two_eb, recip, vmax), lane);
+    wb |= bitlen(__reduce_or_sync(kFull, v[q])) << (8 * q);
+  }
+  return RareOut{v[0], v[1], v[2], v[3], wb, vmax};
 }
 
 // bytes a, b, c, d (each < 256) -> one word, as 3 byte permutes
@@ -969,11 +994,19 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           } else {
             lorenzo_and_counts();
           }
-#ifndef CUSZP_C_EAGER_RARE
+#if !defined(CUSZP_C_EAGER_RARE) && !defined(CUSZP_DIAG_NORARE)
           if (rare) {
+            if constexpr (kScaled && D == 1 && CUSZP_C_RARE_CALL) {
+              const RareOut ro = rare_group_redo(x[0], x[1], x[2], x[3], eb, two_eb, recip, vmax, lane);
+              v[0] = ro.v0; v[1] = ro.v1; v[2] = ro.v2; v[3] = ro.v3;
 #pragma unroll
-            for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
-            lorenzo_and_counts();
+              for (int q = 0; q < 4; ++q) wq[q] = (ro.wb >> (8 * q)) & 0xffu;
+              vmax = ro.vmax;
+            } else {
+#pragma unroll
+              for (int q = 0; q < 4; ++q) r[q] = quantize_exact(x[q], eb, two_eb, recip, vmax);
+              lorenzo_and_counts();
+            }
           }
 #endif
           // room in this warp's ring for a worst-case group (4 x 32 words)
@@ -1024,13 +1057,21 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
             const uint32_t pb = wb * 0x01010100u;                       // exclusive byte prefix (sums <= 24)
             const uint32_t sel = 0x4440u + (uint32_t(lane) >> 3), k = lane & 7;
             if (k < __byte_perm(wb, 0, sel)) ring[(base + __byte_perm(pb, 0, sel) + k) & (kRing - 1)] = tw;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+#ifdef CUSZP_DIAG_NOSPAN32
+          } else {   // diagnostics only: no 1-block-per-transpose path (wrong output when a span > 16)
+#else
           } else if (span <= 16) {
+#endif
             const uint32_t t01 = xpose(__byte_perm(v[0], v[1], 0x5410u));
             const uint32_t t23 = xpose(__byte_perm(v[2], v[3], 0x5410u));
             const bool hi = lane >= 16;
             const uint32_t k = lane & 15;
             if (k < (hi ? wq[1] : wq[0])) ring[(base + (hi ? wq[0] : 0u) + k) & (kRing - 1)] = t01;  // sync: ring slot freed by the writer's tail release; read after staged[m]
             if (k < (hi ? wq[3] : wq[2])) ring[(base + wq[0] + wq[1] + (hi ? wq[2] : 0u) + k) & (kRing - 1)] = t23;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+#ifdef CUSZP_DIAG_NOSPAN32
+          }
+          if (false) {
+#endif
           } else {
             uint32_t o = base;
 #pragma unroll
