@@ -239,6 +239,23 @@ __device__ __forceinline__ uint32_t bitlen(uint32_t x) {
   return p + 1u;
 }
 
+// a group with a block of more than 16 words (span > 16): one transpose per
+// block, words appended to the ring at base (out of line: rare -- none of
+// the bench fields has such a group at the bounds they are run at)
+__device__ __noinline__ void store_singles(uint32_t* ring, uint32_t base, uint32_t v0, uint32_t v1, uint32_t v2,
+                                           uint32_t v3, uint32_t wb, int lane) {
+  const Xpose xpose(lane);
+  const uint32_t v[4] = {v0, v1, v2, v3};
+  uint32_t o = base;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint32_t tq = xpose(v[q]);
+    const uint32_t wq = (wb >> (8 * q)) & 0xffu;
+    if (uint32_t(lane) < wq) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
+    o += wq;
+  }
+}
+
 __device__ __noinline__ RareOut rare_group_redo(float x0, float x1, float x2, float x3, float eb, float two_eb,
                                                 float recip, float vmax, int lane) {
   const float xs[4] = {x0, x1, x2, x3};
@@ -1072,6 +1089,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           }
           if (false) {
 #endif
+          } else if constexpr (CUSZP_C_RARE_CALL && kScaled && D == 1) {
+            store_singles(ring, base, v[0], v[1], v[2], v[3], wb, lane);   // span > 16: rare, out of line
           } else {
             uint32_t o = base;
 #pragma unroll
