@@ -217,9 +217,7 @@ __device__ __forceinline__ uint32_t lorenzo_pack(uint32_t rb, int lane) {
 // hot loop stays compact.  Returns v of the 4 blocks, their word counts
 // (bytes of wb) and the updated guard maximum; 6 values, returned in
 // registers.
-struct RareOut { uint32_t v0, v1, v2, v3, wb; float vmax; };
-__device__ __noinline__ RareOut rare_group_redo(float x0, float x1, float x2, float x3, float eb, float two_eb,
-                                                float recip, float vmax, int lane);
+struct RareOut { uint32_t v0, v1, v2, v3, wb; float vmax; };   // (rare_group_redo: after lorenzo_md_pack)
 
 // same, lane 0 taking `first` (biased) as its predecessor: the last element
 // of the previous 32-element sub-block of an L = 32 M block
@@ -254,18 +252,6 @@ __device__ __noinline__ void store_singles(uint32_t* ring, uint32_t base, uint32
     if (uint32_t(lane) < wq) ring[(o + lane) & (kRing - 1)] = tq;  // sync: ring slot freed by the writer's tail release; read after staged[m]
     o += wq;
   }
-}
-
-__device__ __noinline__ RareOut rare_group_redo(float x0, float x1, float x2, float x3, float eb, float two_eb,
-                                                float recip, float vmax, int lane) {
-  const float xs[4] = {x0, x1, x2, x3};
-  uint32_t v[4], wb = 0;
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    v[q] = lorenzo_pack(quantize_exact(xs[q], eb, two_eb, recip, vmax), lane);
-    wb |= bitlen(__reduce_or_sync(kFull, v[q])) << (8 * q);
-  }
-  return RareOut{v[0], v[1], v[2], v[3], wb, vmax};
 }
 
 // bytes a, b, c, d (each < 256) -> one word, as 3 byte permutes
@@ -358,6 +344,23 @@ __device__ __forceinline__ void block_seq8(const uint32_t* v, uint32_t g, uint32
     s[2] = __byte_perm(hi, hi1, 0x5140u);
     s[3] = __byte_perm(hi, hi1, 0x7362u);
   }
+}
+
+// D = 1: the paper's block Lorenzo; D = 2 / 3: the block-local multi-
+// dimensional predictor (R18), on the integer path like the inline redo
+template <int D>
+__device__ __noinline__ RareOut rare_group_redo(float x0, float x1, float x2, float x3, float eb, float two_eb,
+                                                float recip, float vmax, int lane) {
+  const float xs[4] = {x0, x1, x2, x3};
+  uint32_t v[4], wb = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint32_t r = quantize_exact(xs[q], eb, two_eb, recip, vmax);
+    if constexpr (D == 1) v[q] = lorenzo_pack(r, lane);
+    else v[q] = lorenzo_md_pack<D>(r, lane);
+    wb |= bitlen(__reduce_or_sync(kFull, v[q])) << (8 * q);
+  }
+  return RareOut{v[0], v[1], v[2], v[3], wb, vmax};
 }
 
 // lorenzo_md_pack on SCALED values (quantize_scaled2's r 2^-149): the
@@ -1013,8 +1016,8 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           }
 #if !defined(CUSZP_C_EAGER_RARE) && !defined(CUSZP_DIAG_NORARE)
           if (rare) {
-            if constexpr (kScaled && D == 1 && CUSZP_C_RARE_CALL) {
-              const RareOut ro = rare_group_redo(x[0], x[1], x[2], x[3], eb, two_eb, recip, vmax, lane);
+            if constexpr (kScaled && CUSZP_C_RARE_CALL) {
+              const RareOut ro = rare_group_redo<D>(x[0], x[1], x[2], x[3], eb, two_eb, recip, vmax, lane);
               v[0] = ro.v0; v[1] = ro.v1; v[2] = ro.v2; v[3] = ro.v3;
 #pragma unroll
               for (int q = 0; q < 4; ++q) wq[q] = (ro.wb >> (8 * q)) & 0xffu;
@@ -1089,7 +1092,7 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
           }
           if (false) {
 #endif
-          } else if constexpr (CUSZP_C_RARE_CALL && kScaled && D == 1) {
+          } else if constexpr (CUSZP_C_RARE_CALL && kScaled) {
             store_singles(ring, base, v[0], v[1], v[2], v[3], wb, lane);   // span > 16: rare, out of line
           } else {
             uint32_t o = base;
