@@ -24,6 +24,12 @@
 //               their global offsets and release ring space in tile order.
 //               Up to kMeta tiles wait for their prefix while the compute
 //               warps keep going, so the look-back latency stays hidden.
+//               A segment is copied as unrolled groups of four 32-word
+//               chunks (immediate offsets, one uniform exit test per group).
+// Paths that are rare on real fields -- the R2 redo of a group and a group
+// with a block of more than 16 words -- are out-of-line calls, so the
+// unrolled encode loop stays small (the instruction cache matters, DESIGN
+// sec 8.1).
 // Block lengths L = 64 / 128 (M = L/32 sub-blocks per block) reuse the L = 32
 // encode; L = 8 / 16 (SL) encode one block per LANE (16 consecutive floats
 // per lane: 2 blocks of 8 or 1 of 16) with in-register 8x8 bit transposes
