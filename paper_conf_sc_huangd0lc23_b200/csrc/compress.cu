@@ -260,6 +260,16 @@ __device__ __noinline__ void store_singles(uint32_t* ring, uint32_t base, uint32
   }
 }
 
+// the virtual zero pad (R8) of the last tile's slice of one compute warp
+// (kCBPW x 32 floats of the stage), then the proxy fence for the stage
+template <int NPW>
+__device__ __noinline__ void zero_tail_impl(float* src, uint64_t g0, uint64_t n, int lane) {
+  for (int k = lane; k < NPW; k += 32)
+    if (g0 + k >= n) src[k] = 0.0f;  // sync: own slice of the stage; no TMA rewrites it in this launch
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncwarp();
+}
+
 // bytes a, b, c, d (each < 256) -> one word, as 3 byte permutes
 __device__ __forceinline__ uint32_t pack4(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
   return __byte_perm(__byte_perm(a, b, 0x3240u), __byte_perm(c, d, 0x3240u), 0x5410u);
@@ -804,15 +814,13 @@ __global__ void __launch_bounds__(kCThreads, CUSZP_C_MINBLOCKS) compress_kernel(
         if (t == kSentinel) break;                    // the writers stop on the ticket ring
         const uint64_t g0 = uint64_t(t) * kTileElems + uint64_t(w) * kCBPW * 32;   // first element of the warp
         float* src = &sm.in[s][w * kCBPW * 32];
+        auto zero_tail = [](float* p, uint64_t g, uint64_t n, int l) { zero_tail_impl<kCBPW * 32>(p, g, n, l); };
         if (D == 1 && t == a.num_tiles - 1) {
           // virtual zero pad (R8): the ragged part of the last tile is zeroed in
           // shared memory once, so the encode loop needs no per-element test.
           // (No TMA writes this stage again in this launch: the producer's next
           // ticket is a sentinel; the proxy fence orders it anyway.)
-          for (int k = lane; k < kCBPW * 32; k += 32)
-            if (g0 + k >= a.n) src[k] = 0.0f;  // sync: own slice of the stage; no TMA rewrites it in this launch
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          __syncwarp();
+          zero_tail(src, g0, a.n, lane);                 // out of line: once per launch
         }
         uint32_t cursor = 0;
         // free words in this warp's ring (refreshed only when a worst-case
