@@ -75,7 +75,7 @@ namespace {
 #define CUSZP_C_COPY_UNROLLED 1  // copy-out of a ring segment in unrolled groups of 4 chunks (0: the round-2 loop)
 #endif
 #ifndef CUSZP_C_RARE_CALL
-#define CUSZP_C_RARE_CALL 1      // the R2-correction redo of a group as an out-of-line call (L = 32, 1D, order 1)
+#define CUSZP_C_RARE_CALL 1      // the R2-correction redo and > 16-word stores of a group as out-of-line calls (L = 32, order 1)
 #endif
 #ifndef CUSZP_C_FULL_POLL_NS
 #define CUSZP_C_FULL_POLL_NS 0   // > 0: compute warps poll their input stage with test + nanosleep
@@ -217,8 +217,8 @@ __device__ __forceinline__ uint32_t lorenzo_pack(uint32_t rb, int lane) {
   const uint32_t a = uint32_t(l < 0 ? -l : l);
   return (a << 1) | (uint32_t(l) >> 31);
 }
-// The R2 correction of one group of 4 blocks (L = 32, 1D, order 1), out of
-// line: the rare redo of the unrolled encode loop (an element within an ulp
+// The R2 correction of one group of 4 blocks (L = 32, order 1; 1D or the
+// multi-dimensional predictors), out of line: the rare redo of the unrolled encode loop (an element within an ulp
 // of a half integer of 2eb) as a call instead of four inlined copies, so the
 // hot loop stays compact.  Returns v of the 4 blocks, their word counts
 // (bytes of wb) and the updated guard maximum; 6 values, returned in
