@@ -256,6 +256,7 @@ def container_capacity(shard_n: list[int]) -> int:
 
 
 _peer_cache: dict = {}
+_inflight: list = []     # (IPC view, event): mappings kept alive until the puts through them completed
 
 
 def _peer_view(buf: torch.Tensor | None, dst: int, group, cache_key=None) -> torch.Tensor:
@@ -304,6 +305,12 @@ def gather_container_p2p(res: ShardResult, shard_n: list[int], group=None, dst: 
         if _nccl(group):
             tok = torch.zeros(1, dtype=torch.int32, device=dev)
             dist.all_reduce(tok, group=group)                # after every put on every rank's stream
+            if rank != dst and cache_key is None:
+                # the put is still queued: keep the IPC mapping alive until it ran
+                ev = torch.cuda.Event()
+                ev.record(s)
+                _inflight.append((view, ev))
+                _inflight[:] = [(v, e) for v, e in _inflight if not e.query()]
         else:
             torch.cuda.synchronize(dev)                      # gloo (tests): host-ordered
             dist.barrier(group=group)
