@@ -782,10 +782,15 @@ def run_ours(args, rank, world, dev):
     line["quality"] = verify(r, jobs)
 
     if not args.no_e2e:
+        prev, placement = (bind_to_gpu_numa(dev.index) if os.environ.get("CUSZP_E2E_NUMA", "1") == "1"
+                           else (None, "not bound (CUSZP_E2E_NUMA=0)"))
         hx = {}
         h_jobs = [(lab, hx.setdefault(id(x), x.cpu().pin_memory()), rel) for lab, x, _, rel in jobs]
         line["e2e"] = e2e_measure(cz, dev, h_jobs, K, world, r.cap, nmax)
+        line["e2e"]["host_placement"] = placement
         del h_jobs, hx
+        if prev is not None:
+            os.sched_setaffinity(0, prev)        # the CPU baseline may use every core again
 
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         lab, x, n, rel = jobs[len(jobs) // 2]
@@ -808,6 +813,27 @@ def run_ours(args, rank, world, dev):
     if world == 1 and not args.no_datasets:
         line["datasets"] = datasets_table(peak, 3, dev)
     return line
+
+
+def bind_to_gpu_numa(dev_index: int):
+    """Pin this process to the CPUs local to the GPU (NVML's affinity mask,
+    intersected with the CPUs we may use), so pinned host buffers are first
+    touched -- and allocated -- on the GPU's NUMA node, as a serving process
+    would be placed.  Returns (previous CPU set, description) or (None, why)."""
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+        words = pynvml.nvmlDeviceGetCpuAffinity(h, (os.cpu_count() + 63) // 64)
+        local = {64 * i + b for i, w in enumerate(words) for b in range(64) if (int(w) >> b) & 1}
+        allowed = os.sched_getaffinity(0)
+        cpus = local & allowed
+        if not cpus or cpus == allowed:
+            return None, f"not bound ({len(local)} GPU-local CPUs, {len(allowed)} allowed)"
+        os.sched_setaffinity(0, cpus)
+        return allowed, f"bound to the {len(cpus)} GPU-local CPUs of {len(allowed)}"
+    except Exception as e:  # no NVML / no affinity support: leave the placement alone
+        return None, f"not bound ({type(e).__name__})"
 
 
 def main():
